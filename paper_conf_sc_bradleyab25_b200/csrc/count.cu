@@ -1,0 +1,535 @@
+// count.cu -- fsgc_count: the data-parallel hot path of Fringe-SGC on sm_100a.
+//
+// PAPER.md Sec. 3.3-3.6 and Listing 5 (Fig. 5), Listing 7:
+//   * core matching: depth-first search for the core from each root item
+//     (root edge (c0,c1) or root vertex), one warp per root, the warp-ballot
+//     scheme of Listing 7 ("the 32 warp threads concurrently process 32
+//     vertices ... all lanes process the first such vertex together"),
+//     symmetry breaking on degree-ordered ids (Sec. 3.1), degree filtering;
+//   * Venn diagram: for each anchor vertex, the warp scans its sorted
+//     adjacency list and binary-searches the anchors later in the order
+//     (Sec. 3.6 "we search the adjacency lists of the anchor vertices that
+//     appear later in the stack ... with binary search"), histograms the
+//     membership bitsets, then corrects the counts for the earlier anchors and
+//     excludes the matched core vertices;
+//   * fringe counting: up to 32 Venn diagrams are buffered per warp, then the
+//     lanes evaluate the iterative form of Listing 5 on (diagram, program)
+//     pairs ("each lane runs the iterative fc function");
+//   * exact 128-bit accumulation, warp-shuffle reduction, one 128-bit atomic
+//     per warp and pattern.
+// Work distribution: persistent CTAs, a global atomic chunk queue, heavy
+// (high-degree, late in degree order) roots handed out first; shards deal
+// chunks round-robin across GPUs.
+#include <algorithm>
+#include <cstring>
+#include "devbuf.cuh"
+#include "u128.cuh"
+
+#define FULLMASK 0xffffffffu
+
+namespace {
+
+struct GraphDev {
+    const int64_t* __restrict__ offs;
+    const int32_t* __restrict__ adj;
+    const int32_t* __restrict__ row;
+    const int32_t* __restrict__ osrc;
+    const int32_t* __restrict__ odst;
+};
+
+struct WorkDesc {
+    int64_t begin, end;   // root item range
+    int32_t shard, nshards;
+    int32_t chunk;        // items per queue grab
+    int32_t degfilter;    // 1: apply the degree filter
+};
+
+struct AccDev {
+    unsigned long long lo, hi;
+    unsigned int ovf, pad;
+    unsigned long long pad2;
+};
+
+__device__ __forceinline__ bool contains(const int32_t* __restrict__ L, int len, int x) {
+    int lo = 0, hi = len;
+    while (lo < hi) {
+        int mid = (lo + hi) >> 1;
+        if (__ldg(L + mid) < x) lo = mid + 1; else hi = mid;
+    }
+    return lo < len && __ldg(L + lo) == x;
+}
+
+// first index with L[i] > x
+__device__ __forceinline__ int upper_bound(const int32_t* __restrict__ L, int len, int x) {
+    int lo = 0, hi = len;
+    while (lo < hi) {
+        int mid = (lo + hi) >> 1;
+        if (__ldg(L + mid) <= x) lo = mid + 1; else hi = mid;
+    }
+    return lo;
+}
+
+struct Frame {
+    u128 M;
+    uint32_t vc;
+    uint8_t pos, rem, idx, i, top, kind;
+};
+
+// Iterative Listing 5: the recursion fc(pos, rem, idx) with an explicit
+// stack.  `venn` is this lane's private copy; it is decremented/restored
+// exactly as lines 10/12 and 18/20 of the listing do.
+__device__ u128 fc_eval(uint32_t* venn, int q, const FringeProg& P, bool& ovf) {
+    const int s = P.s;
+    if (s == 0) return 1;
+    const int full = (1 << q) - 1;
+    Frame st[FSGC_FC_STACK];
+    int sp = 0;
+    u128 total = 0;
+    int pos = 0, rem = P.k[0], idx = P.anch[0];
+    u128 M = 1;
+    for (;;) {
+        // ---- enter fc(pos, rem, idx) with multiplier M
+        for (;;) {
+            if (rem == 0) {                              // line 6: next type
+                if (++pos == s) { total = add_ovf(total, M, ovf); break; }  // line 5
+                rem = P.k[pos];
+                idx = P.anch[pos];
+                continue;
+            }
+            const uint32_t vc = venn[idx];               // line 7
+            if (idx == full) {                           // line 8: last entry
+                if ((uint32_t)rem > vc) break;           // line 9: no solution
+                M = mul_ovf(M, binom_ovf(vc, (uint32_t)rem, ovf), ovf);  // line 11
+                venn[idx] = vc - rem;                    // line 10
+                Frame f;
+                f.kind = 0; f.idx = (uint8_t)idx; f.rem = (uint8_t)rem;
+                st[sp++] = f;
+                rem = 0;
+                continue;
+            }
+            const int top = min(rem, (int)vc);           // line 16
+            Frame f;
+            f.M = M; f.vc = vc; f.pos = (uint8_t)pos; f.rem = (uint8_t)rem;
+            f.idx = (uint8_t)idx; f.i = 0; f.top = (uint8_t)top; f.kind = 1;
+            st[sp++] = f;                                 // i = 0: C(vc,0) = 1
+            idx = (idx + 1) | P.anch[pos];               // line 19: next entry
+        }
+        // ---- return: undo and advance the innermost open summation
+        for (;;) {
+            if (sp == 0) return total;
+            Frame& f = st[sp - 1];
+            if (f.kind == 0) { venn[f.idx] += f.rem; --sp; continue; }  // line 12
+            venn[f.idx] += f.i;                          // line 20
+            if (++f.i > f.top) { --sp; continue; }
+            venn[f.idx] -= f.i;                          // line 18
+            M = mul_ovf(f.M, binom_ovf(f.vc, f.i, ovf), ovf);
+            pos = f.pos;
+            rem = f.rem - f.i;
+            idx = (f.idx + 1) | P.anch[f.pos];
+            break;
+        }
+    }
+}
+
+__device__ __forceinline__ void warp_reduce_u128(u128& v, bool& ovf) {
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        uint64_t lo = __shfl_down_sync(FULLMASK, u128_lo(v), o);
+        uint64_t hi = __shfl_down_sync(FULLMASK, u128_hi(v), o);
+        int f = __shfl_down_sync(FULLMASK, (int)ovf, o);
+        v = add_ovf(v, u128_make(lo, hi), ovf);
+        ovf |= (f != 0);
+    }
+}
+
+__device__ __forceinline__ void atomic_add_u128(AccDev* a, u128 v, bool ovf) {
+    const uint64_t lo = u128_lo(v), hi = u128_hi(v);
+    bool o = ovf;
+    uint64_t carry = 0;
+    if (lo) {
+        unsigned long long old = atomicAdd(&a->lo, (unsigned long long)lo);
+        carry = (old + lo < old) ? 1 : 0;
+    }
+    uint64_t hadd = hi + carry;
+    if (hadd < hi) o = true;
+    if (hadd) {
+        unsigned long long oldh = atomicAdd(&a->hi, (unsigned long long)hadd);
+        if (oldh + hadd < oldh) o = true;
+    }
+    if (o) atomicOr(&a->ovf, 1u);
+}
+
+// per-warp epilogue: reduce the lane accumulators, one atomic per pattern
+__device__ __forceinline__ void warp_flush_acc(int npats, u128* acc_l, bool ovf, unsigned long long nmatch,
+                                               AccDev* acc, unsigned long long* matches, int lane) {
+    for (int pi = 0; pi < npats; ++pi) {
+        u128 v = acc_l[pi];
+        bool o = ovf;
+        warp_reduce_u128(v, o);
+        if (lane == 0 && (v != 0 || o)) atomic_add_u128(acc + pi, v, o);
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) nmatch += __shfl_down_sync(FULLMASK, nmatch, o);
+    if (lane == 0 && nmatch) atomicAdd(matches, nmatch);
+}
+
+// ------------------------------------------------------------------------
+// 1-vertex cores (k-stars, the 1- and 2-vertex patterns): one thread per
+// root vertex, Venn = {deg(v)} (Sec. 3 k-star formula generalised by fc).
+__global__ void __launch_bounds__(256) vertex_core_kernel(GraphDev G, const CoreProg P, WorkDesc W,
+                                                          AccDev* acc, unsigned long long* matches) {
+    const int lane = threadIdx.x & 31;
+    u128 acc_l[FSGC_MAXPATS];
+    for (int i = 0; i < FSGC_MAXPATS; ++i) acc_l[i] = 0;
+    bool ovf = false;
+    unsigned long long nmatch = 0;
+    const int64_t total = W.end - W.begin;
+    const int64_t nchunks = (total + W.chunk - 1) / W.chunk;
+    const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    const int64_t nthreads = (int64_t)gridDim.x * blockDim.x;
+    // chunk c of this shard = global chunk c * nshards + shard
+    for (int64_t c = tid / W.chunk; ; c += nthreads / W.chunk) {
+        int64_t g = c * W.nshards + W.shard;
+        if (g >= nchunks) break;
+        int64_t t = g * W.chunk + tid % W.chunk;
+        if (t >= total) continue;
+        const int64_t v = W.begin + t;
+        const uint32_t deg = (uint32_t)(G.offs[v + 1] - G.offs[v]);
+        if (W.degfilter && (int)deg < P.mindeg[0]) continue;
+        ++nmatch;
+        uint32_t venn[2] = {0, deg};
+        for (int pi = 0; pi < P.nprog; ++pi) {
+            const FringeProg fp = P.prog[pi];
+            u128 c2 = fc_eval(venn, P.q, fp, ovf);
+            acc_l[fp.pat] = add_ovf(acc_l[fp.pat], c2, ovf);
+        }
+    }
+    warp_flush_acc(P.npats, acc_l, ovf, nmatch, acc, matches, lane);
+}
+
+// ------------------------------------------------------------------------
+// Cores with p >= 2 vertices: one warp per root edge.
+template <int WARPS>
+__global__ void __launch_bounds__(WARPS * 32) core_kernel(GraphDev G, const CoreProg P, WorkDesc W,
+                                                          AccDev* acc, unsigned long long* matches,
+                                                          unsigned long long* queue) {
+    extern __shared__ uint32_t smem[];
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    const int q = P.q, V = 1 << q, p = P.p;
+    uint32_t* hist = smem + wib * (V * 33);
+    uint32_t* vbuf = hist + V;
+    int nbuf = 0;
+    u128 acc_l[FSGC_MAXPATS];
+    for (int i = 0; i < FSGC_MAXPATS; ++i) acc_l[i] = 0;
+    bool ovf = false;
+    unsigned long long nmatch = 0;
+
+    int emb[FSGC_MAXC];
+    int64_t eoff[FSGC_MAXC];
+    int edeg[FSGC_MAXC];
+    int64_t cur[FSGC_MAXC], endp[FSGC_MAXC];
+    int pivl[FSGC_MAXC];
+    uint32_t pend[FSGC_MAXC];
+
+    // ---- fc over the buffered Venn diagrams, lanes over (diagram, program)
+    auto flush = [&]() {
+        __syncwarp();
+        const int tot = nbuf * P.nprog;
+        for (int t = lane; t < tot; t += 32) {
+            const int vi = t / P.nprog, pi = t - vi * P.nprog;
+            uint32_t vloc[1 << FSGC_MAXQ];
+            for (int e = 0; e < V; ++e) vloc[e] = vbuf[vi * V + e];
+            const FringeProg fp = P.prog[pi];
+            u128 c = fc_eval(vloc, q, fp, ovf);
+            acc_l[fp.pat] = add_ovf(acc_l[fp.pat], c, ovf);
+        }
+        nbuf = 0;
+        __syncwarp();
+    };
+
+    // ---- Venn diagram of the current core match into vbuf[nbuf]
+    auto leaf = [&]() {
+        if (lane == 0) ++nmatch;
+        uint32_t* R = vbuf + nbuf * V;
+        for (int t = lane; t < V; t += 32) hist[t] = 0;
+        __syncwarp();
+        for (int i = 0; i < q; ++i) {
+            const int pi = P.anchor_pos[i];
+            const int32_t* __restrict__ Li = G.adj + eoff[pi];
+            const int li = edeg[pi];
+            for (int b0 = 0; b0 < li; b0 += 32) {
+                const int ix = b0 + lane;
+                bool valid = ix < li;
+                const int x = valid ? __ldg(Li + ix) : -1;
+#pragma unroll
+                for (int j = 0; j < FSGC_MAXC; ++j)
+                    if (j < p && x == emb[j]) valid = false;   // e(x) excludes the core
+                uint32_t m = 1u << i;
+                if (valid)
+                    for (int j = i + 1; j < q; ++j) {
+                        const int pj = P.anchor_pos[j];
+                        if (contains(G.adj + eoff[pj], edeg[pj], x)) m |= 1u << j;
+                    }
+                const unsigned act = __ballot_sync(FULLMASK, valid);
+                if (valid) {
+                    const unsigned peers = __match_any_sync(act, m);
+                    if (lane == __ffs(peers) - 1) hist[m] += __popc(peers);
+                }
+                __syncwarp();
+            }
+        }
+        // regions: entries whose lowest bit is i are exact once the regions
+        // with a lower lowest bit are known (Sec. 3.6 "we computationally
+        // correct them")
+        for (int i = 0; i < q; ++i) {
+            for (int t = lane; t < V; t += 32) {
+                if (t == 0 || (__ffs(t) - 1) != i) continue;
+                int r = (int)hist[t];
+                const int low = (1 << i) - 1;
+                for (int E = low; E > 0; E = (E - 1) & low) r -= (int)R[E | t];
+                R[t] = (uint32_t)r;
+            }
+            __syncwarp();
+        }
+        if (lane == 0) R[0] = 0;
+        __syncwarp();
+        if (++nbuf == 32) flush();
+    };
+
+    auto init_level = [&](int l) {
+        int piv = -1, best = 0x7fffffff;
+#pragma unroll
+        for (int j = 0; j < FSGC_MAXC; ++j)
+            if (j < l && (P.back[l] >> j & 1) && edeg[j] < best) { best = edeg[j]; piv = j; }
+        int64_t b = eoff[piv], e = eoff[piv] + edeg[piv];
+        if (P.gt[l]) {
+            int lb = -1;
+#pragma unroll
+            for (int j = 0; j < FSGC_MAXC; ++j)
+                if (j < l && (P.gt[l] >> j & 1)) lb = max(lb, emb[j]);
+            b += upper_bound(G.adj + b, (int)(e - b), lb);
+        }
+        cur[l] = b;
+        endp[l] = e;
+        pend[l] = 0;
+        pivl[l] = piv;
+    };
+
+    const int64_t total = W.end - W.begin;
+    for (;;) {
+        unsigned long long jq = 0;
+        if (lane == 0) jq = atomicAdd(queue, 1ull);
+        jq = __shfl_sync(FULLMASK, jq, 0);
+        const int64_t g = (int64_t)jq * W.nshards + W.shard;
+        const int64_t t0 = g * W.chunk;
+        if (t0 >= total) break;
+        const int64_t t1 = min(t0 + (int64_t)W.chunk, total);
+        for (int64_t t = t0; t < t1; ++t) {
+            const int64_t item = W.end - 1 - t;   // heavy roots first
+            int u0, u1;
+            if (P.root_mode == ROOT_ORIENTED) { u0 = __ldg(G.osrc + item); u1 = __ldg(G.odst + item); }
+            else { u0 = __ldg(G.row + item); u1 = __ldg(G.adj + item); }
+            emb[0] = u0; eoff[0] = G.offs[u0]; edeg[0] = (int)(G.offs[u0 + 1] - eoff[0]);
+            emb[1] = u1; eoff[1] = G.offs[u1]; edeg[1] = (int)(G.offs[u1 + 1] - eoff[1]);
+            if (W.degfilter && (edeg[0] < P.mindeg[0] || edeg[1] < P.mindeg[1])) continue;
+            if (p == 2) { leaf(); continue; }
+            int lvl = 2;
+            init_level(2);
+            while (lvl >= 2) {
+                if (pend[lvl] == 0) {
+                    if (cur[lvl] >= endp[lvl]) { --lvl; continue; }
+                    const int64_t pidx = cur[lvl] + lane;
+                    bool ok = pidx < endp[lvl];
+                    const int x = ok ? __ldg(G.adj + pidx) : -1;
+                    if (ok) {
+#pragma unroll
+                        for (int j = 0; j < FSGC_MAXC; ++j)
+                            if (j < lvl && (x == emb[j] || ((P.gt[lvl] >> j & 1) && x <= emb[j]))) ok = false;
+                    }
+                    if (ok && W.degfilter) ok = (int)(G.offs[x + 1] - G.offs[x]) >= P.mindeg[lvl];
+                    if (ok) {
+                        const int piv = pivl[lvl];
+                        for (int j = 0; j < lvl && ok; ++j)
+                            if ((P.back[lvl] >> j & 1) && j != piv)
+                                ok = contains(G.adj + eoff[j], edeg[j], x);
+                    }
+                    pend[lvl] = __ballot_sync(FULLMASK, ok);
+                    cur[lvl] += 32;   // candidates are re-read from adj[cur - 32 + who]
+                    continue;
+                }
+                const int who = __ffs(pend[lvl]) - 1;
+                pend[lvl] &= pend[lvl] - 1;
+                const int x = __ldg(G.adj + (cur[lvl] - 32) + who);
+                emb[lvl] = x;
+                eoff[lvl] = G.offs[x];
+                edeg[lvl] = (int)(G.offs[x + 1] - eoff[lvl]);
+                if (lvl == p - 1) {
+                    leaf();
+                } else {
+                    ++lvl;
+                    init_level(lvl);
+                }
+            }
+        }
+    }
+    if (nbuf) flush();
+    warp_flush_acc(P.npats, acc_l, ovf, nmatch, acc, matches, lane);
+}
+
+int sm_count() {
+    static int n = 0;
+    if (!n) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+        if (n <= 0) n = 148;
+    }
+    return n;
+}
+
+constexpr int kWarps = 4;
+
+}  // namespace
+
+static int64_t roots_for(const fsgc_graph* g, int root_mode) {
+    switch (root_mode) {
+        case ROOT_VERTEX: return g->n;
+        case ROOT_ORIENTED: return g->m;
+        default: return 2 * g->m;
+    }
+}
+
+extern "C" int fsgc_finalize(fsgc_u128 raw, uint64_t divisor, int32_t overflow, fsgc_u128* count,
+                             int32_t* count_overflow) {
+    if (!count || !count_overflow || divisor == 0) FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_finalize: bad argument");
+    u128 r = u128_make(raw.lo, raw.hi);
+    if (!overflow && (r % divisor) != 0)
+        FSGC_FAIL(FSGC_ERR_INTERNAL, "raw sum not divisible by the automorphism divisor");
+    u128 c = r / divisor;
+    count->lo = u128_lo(c);
+    count->hi = u128_hi(c);
+    *count_overflow = overflow ? 1 : 0;
+    return FSGC_OK;
+}
+
+// group patterns with isomorphic cores (one pass each)
+static std::vector<std::vector<int>> group_patterns(const fsgc_pattern* const* pats, int npats) {
+    std::vector<std::vector<int>> groups;
+    int pos_of[FSGC_MAX_PATTERN_VERTICES];
+    for (int i = 0; i < npats; ++i) {
+        bool placed = false;
+        for (auto& gr : groups)
+            if (fsgc_core_isomorphism(pats[gr[0]], pats[i], pos_of)) { gr.push_back(i); placed = true; break; }
+        if (!placed) groups.push_back({i});
+    }
+    return groups;
+}
+
+extern "C" int fsgc_num_roots(const fsgc_graph* g, const fsgc_pattern* p, int nosym, int64_t* out) {
+    if (!g || !p || !out) FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_num_roots: null argument");
+    PassPlan plan;
+    std::vector<int> mem{0};
+    const fsgc_pattern* arr[1] = {p};
+    int rc = fsgc_build_pass(arr, mem, nosym, &plan);
+    if (rc) return rc;
+    *out = roots_for(g, plan.prog.root_mode);
+    return FSGC_OK;
+}
+
+extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, int npats,
+                          const fsgc_count_opts* opts_in, fsgc_result* results, void* stream_) {
+    if (!g || !pats || !results || npats < 1 || npats > FSGC_MAX_BATCH)
+        FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_count: bad arguments");
+    for (int i = 0; i < npats; ++i)
+        if (!pats[i]) FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_count: null pattern %d", i);
+    fsgc_count_opts opts{0, -1, 0, 1, 0, 0};
+    if (opts_in) opts = *opts_in;
+    if (opts.shard_count < 1 || opts.shard_index < 0 || opts.shard_index >= opts.shard_count)
+        FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_count: bad shard %d/%d", opts.shard_index, opts.shard_count);
+    cudaStream_t st = (cudaStream_t)stream_;
+    std::memset(results, 0, sizeof(fsgc_result) * npats);
+
+    auto groups = group_patterns(pats, npats);
+    for (auto& members : groups) {
+        PassPlan plan;
+        int rc = fsgc_build_pass(pats, members, opts.no_symmetry_breaking, &plan);
+        if (rc) return rc;
+        const CoreProg& cp = plan.prog;
+        const int64_t R = roots_for(g, cp.root_mode);
+        int64_t b = opts.root_begin < 0 ? 0 : opts.root_begin;
+        int64_t e = (opts.root_end < 0 || opts.root_end > R) ? R : opts.root_end;
+        if (b > e) b = e;
+
+        const int npm = (int)members.size();
+        DevBuf<unsigned char> scratch;
+        const size_t acc_bytes = sizeof(AccDev) * FSGC_MAXPATS;
+        FSGC_CUDA(scratch.alloc(acc_bytes + 64, st));
+        AccDev* dacc = (AccDev*)scratch.ptr;
+        unsigned long long* dmatch = (unsigned long long*)(scratch.ptr + acc_bytes);
+        unsigned long long* dqueue = dmatch + 1;
+        FSGC_CUDA(cudaMemsetAsync(scratch.ptr, 0, acc_bytes + 64, st));
+
+        GraphDev G{g->offsets, g->adj, g->row, g->osrc, g->odst};
+        WorkDesc W{b, e, opts.shard_index, opts.shard_count, 4,
+                   (opts.flags & FSGC_FLAG_NO_DEGREE_FILTER) ? 0 : 1};
+        static thread_local cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+        if (!ev0) {
+            FSGC_CUDA(cudaEventCreate(&ev0));
+            FSGC_CUDA(cudaEventCreate(&ev1));
+        }
+        int launches = 0;
+        FSGC_CUDA(cudaEventRecord(ev0, st));
+        if (e > b) {
+            launches = 1;
+            if (cp.root_mode == ROOT_VERTEX) {
+                W.chunk = 256;
+                int64_t work = (e - b + opts.shard_count - 1) / opts.shard_count;
+                int64_t grid = (work + 255) / 256;
+                grid = std::max<int64_t>(1, std::min<int64_t>(grid, (int64_t)sm_count() * 8));
+                vertex_core_kernel<<<(int)grid, 256, 0, st>>>(G, cp, W, dacc, dmatch);
+                FSGC_CUDA(cudaGetLastError());
+            } else {
+                const size_t smem = (size_t)kWarps * 33 * (1u << cp.q) * sizeof(uint32_t);
+                static bool attr_set = false;
+                if (!attr_set) {
+                    FSGC_CUDA(cudaFuncSetAttribute(core_kernel<kWarps>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                   (int)(kWarps * 33 * (1u << FSGC_MAXQ) * sizeof(uint32_t))));
+                    attr_set = true;
+                }
+                int per_sm = 0;
+                FSGC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, core_kernel<kWarps>, kWarps * 32, smem));
+                if (per_sm < 1) per_sm = 1;
+                int64_t nchunks = ((e - b) + W.chunk - 1) / W.chunk;
+                int64_t mine = (nchunks + opts.shard_count - 1) / opts.shard_count;
+                int64_t grid = std::min<int64_t>((int64_t)sm_count() * per_sm, (mine + kWarps - 1) / kWarps);
+                if (grid < 1) grid = 1;
+                core_kernel<kWarps><<<(int)grid, kWarps * 32, smem, st>>>(G, cp, W, dacc, dmatch, dqueue);
+                FSGC_CUDA(cudaGetLastError());
+            }
+        }
+        FSGC_CUDA(cudaEventRecord(ev1, st));
+        AccDev hacc[FSGC_MAXPATS];
+        unsigned long long hmatch = 0;
+        FSGC_CUDA(cudaMemcpyAsync(hacc, dacc, acc_bytes, cudaMemcpyDeviceToHost, st));
+        FSGC_CUDA(cudaMemcpyAsync(&hmatch, dmatch, sizeof hmatch, cudaMemcpyDeviceToHost, st));
+        FSGC_CUDA(cudaStreamSynchronize(st));
+        float kms = 0.f;
+        FSGC_CUDA(cudaEventElapsedTime(&kms, ev0, ev1));
+        for (int mi = 0; mi < npm; ++mi) {
+            fsgc_result& r = results[members[mi]];
+            r.raw.lo = hacc[mi].lo;
+            r.raw.hi = hacc[mi].hi;
+            r.overflow = hacc[mi].ovf ? 1 : 0;
+            r.divisor = plan.divisor[mi];
+            r.core_matches = hmatch;
+            r.root_pattern_vertex = plan.root_pattern_vertex[mi];
+            r.kernel_ms = kms;
+            r.kernel_launches = launches;
+            if (opts.shard_count == 1 && opts.root_begin <= 0 && opts.root_end < 0) {
+                rc = fsgc_finalize(r.raw, r.divisor, r.overflow, &r.count, &r.overflow);
+                if (rc) return rc;
+            }
+        }
+    }
+    return FSGC_OK;
+}

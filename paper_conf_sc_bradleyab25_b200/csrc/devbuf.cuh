@@ -1,0 +1,43 @@
+// devbuf.cuh -- stream-ordered device allocations with RAII + error macros.
+#pragma once
+#include <cuda_runtime.h>
+#include "internal.h"
+
+#define FSGC_CUDA(call)                                                              \
+    do {                                                                             \
+        cudaError_t e_ = (call);                                                     \
+        if (e_ != cudaSuccess) {                                                     \
+            fsgc_set_error("%s failed: %s (%s:%d)", #call, cudaGetErrorString(e_),   \
+                           __FILE__, __LINE__);                                      \
+            return e_ == cudaErrorMemoryAllocation ? FSGC_ERR_OOM : FSGC_ERR_CUDA;   \
+        }                                                                            \
+    } while (0)
+
+template <typename T>
+struct DevBuf {
+    T* ptr = nullptr;
+    size_t count = 0;
+    cudaStream_t stream = nullptr;
+    DevBuf() = default;
+    DevBuf(const DevBuf&) = delete;
+    DevBuf& operator=(const DevBuf&) = delete;
+    ~DevBuf() { release(); }
+    cudaError_t alloc(size_t n, cudaStream_t s) {
+        release();
+        stream = s;
+        count = n;
+        if (n == 0) return cudaSuccess;
+        return cudaMallocAsync((void**)&ptr, n * sizeof(T), s);
+    }
+    void release() {
+        if (ptr) cudaFreeAsync(ptr, stream);
+        ptr = nullptr;
+        count = 0;
+    }
+    T* take() {  // transfer ownership out
+        T* p = ptr;
+        ptr = nullptr;
+        count = 0;
+        return p;
+    }
+};

@@ -1,0 +1,317 @@
+// graph.cu -- fsgc_load_graph: edge list -> deduplicated, symmetrised,
+// degree-ordered CSR in HBM (north_star; Sec. 2 undirected simple
+// graphs, Sec. 3.6 degree-based matching order / symmetry breaking on ids).
+//
+// Device pipeline (all on `stream`, sorts/compaction via CUB, the rest here):
+//   1 emit    each input edge (a,b), a != b  ->  keys a<<B|b and b<<B|a
+//             (B = bits to hold n-1); loops / out-of-range -> sentinel
+//   2 sort    radix sort on the low 2B bits; 3 unique (dedup directed pairs)
+//   4 degree  per-vertex lower_bound into the sorted keys
+//   5 order   sort (deg<<B | id) -> new id = rank (degree asc, id asc)
+//   6 relabel keys -> rank[a]<<B | rank[b]; radix sort again
+//   7 CSR     adj/row = key halves, offsets = exclusive scan of new degrees,
+//             oriented edges (u < v) = compaction of the upper triangle
+// HBM layout of the result: offsets int64[n+1], adj int32[2m], row int32[2m],
+// osrc/odst int32[m] (SoA, sorted by (u, v)), order int32[n].
+#include <cub/cub.cuh>
+#include "devbuf.cuh"
+
+namespace {
+
+__global__ void emit_keys(const void* __restrict__ edges, int64_t E, int ib, int64_t n, int B,
+                          uint64_t sentinel, uint64_t* __restrict__ keys, int* __restrict__ bad) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < E;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        int64_t a, b;
+        if (ib == 4) {
+            const int32_t* e = reinterpret_cast<const int32_t*>(edges);
+            a = e[2 * i]; b = e[2 * i + 1];
+        } else {
+            const int64_t* e = reinterpret_cast<const int64_t*>(edges);
+            a = e[2 * i]; b = e[2 * i + 1];
+        }
+        uint64_t k0 = sentinel, k1 = sentinel;
+        if (a < 0 || b < 0 || a >= n || b >= n) {
+            *bad = 1;
+        } else if (a != b) {
+            k0 = ((uint64_t)a << B) | (uint64_t)b;
+            k1 = ((uint64_t)b << B) | (uint64_t)a;
+        }
+        keys[2 * i] = k0;
+        keys[2 * i + 1] = k1;
+    }
+}
+
+// offs[v] = first index i with (keys[i] >> B) >= v, for v in [0, n]
+__global__ void lower_bounds(const uint64_t* __restrict__ keys, int64_t M, int64_t n, int B,
+                             int64_t* __restrict__ offs) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v <= n;
+         v += (int64_t)gridDim.x * blockDim.x) {
+        uint64_t target = (uint64_t)v << B;
+        int64_t lo = 0, hi = M;
+        while (lo < hi) {
+            int64_t mid = (lo + hi) >> 1;
+            if (keys[mid] < target) lo = mid + 1; else hi = mid;
+        }
+        offs[v] = lo;
+    }
+}
+
+__global__ void degree_keys(const int64_t* __restrict__ offs, int64_t n, int B, uint64_t* __restrict__ vk) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
+         v += (int64_t)gridDim.x * blockDim.x)
+        vk[v] = ((uint64_t)(offs[v + 1] - offs[v]) << B) | (uint64_t)v;
+}
+
+__global__ void ranks_from_order(const uint64_t* __restrict__ vk, int64_t n, int B,
+                                 int32_t* __restrict__ order, int32_t* __restrict__ rank,
+                                 int64_t* __restrict__ deg_new) {
+    const uint64_t mask = (1ull << B) - 1;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        uint64_t k = vk[i];
+        int32_t v = (int32_t)(k & mask);
+        order[i] = v;
+        rank[v] = (int32_t)i;
+        deg_new[i] = (int64_t)(k >> B);
+    }
+}
+
+__global__ void relabel_keys(uint64_t* __restrict__ keys, int64_t M, int B, const int32_t* __restrict__ rank) {
+    const uint64_t mask = (1ull << B) - 1;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < M;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        uint64_t k = keys[i];
+        uint64_t a = (uint64_t)rank[k >> B], b = (uint64_t)rank[k & mask];
+        keys[i] = (a << B) | b;
+    }
+}
+
+__global__ void split_keys(const uint64_t* __restrict__ keys, int64_t M, int B,
+                           int32_t* __restrict__ row, int32_t* __restrict__ adj) {
+    const uint64_t mask = (1ull << B) - 1;
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < M;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        uint64_t k = keys[i];
+        row[i] = (int32_t)(k >> B);
+        adj[i] = (int32_t)(k & mask);
+    }
+}
+
+struct UpperTri {
+    int B;
+    uint64_t mask;
+    __host__ __device__ bool operator()(const uint64_t& k) const { return (k >> B) < (k & mask); }
+};
+
+int grid_for(int64_t work) {
+    int64_t g = (work + 255) / 256;
+    if (g > 148 * 32) g = 148 * 32;
+    if (g < 1) g = 1;
+    return (int)g;
+}
+
+}  // namespace
+
+extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, int on_device,
+                               void* stream_, fsgc_graph** out) {
+    if (!out) FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_load_graph: out is NULL");
+    *out = nullptr;
+    if (E < 0 || (E > 0 && !edges)) FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_load_graph: bad edge list");
+    if (ib != 4 && ib != 8) FSGC_FAIL(FSGC_ERR_INVALID, "index_bytes must be 4 or 8");
+    if (n <= 0 || n >= (1ll << 31)) FSGC_FAIL(FSGC_ERR_INVALID, "num_vertices must be in [1, 2^31)");
+    cudaStream_t st = (cudaStream_t)stream_;
+    int dev = 0;
+    FSGC_CUDA(cudaGetDevice(&dev));
+
+    int B = 1;
+    while ((1ll << B) < n) ++B;
+    const int keybits = 2 * B;
+    const uint64_t sentinel = (keybits == 64) ? ~0ull : ((1ull << keybits) - 1);
+
+    // 1 emit
+    DevBuf<char> din;
+    const void* dedges = edges;
+    if (!on_device && E > 0) {
+        FSGC_CUDA(din.alloc((size_t)E * 2 * ib, st));
+        FSGC_CUDA(cudaMemcpyAsync(din.ptr, edges, (size_t)E * 2 * ib, cudaMemcpyHostToDevice, st));
+        dedges = din.ptr;
+    }
+    const int64_t K = 2 * E;
+    DevBuf<uint64_t> ka, kb;
+    DevBuf<int> dbad;
+    FSGC_CUDA(ka.alloc(K > 0 ? K : 1, st));
+    FSGC_CUDA(kb.alloc(K > 0 ? K : 1, st));
+    FSGC_CUDA(dbad.alloc(1, st));
+    FSGC_CUDA(cudaMemsetAsync(dbad.ptr, 0, sizeof(int), st));
+    if (E > 0) {
+        emit_keys<<<grid_for(E), 256, 0, st>>>(dedges, E, ib, n, B, sentinel, ka.ptr, dbad.ptr);
+        FSGC_CUDA(cudaGetLastError());
+    }
+    din.release();
+
+    // 2 sort, 3 unique
+    DevBuf<char> tmp;
+    size_t tmp_bytes = 0;
+    DevBuf<int64_t> dnum;
+    FSGC_CUDA(dnum.alloc(1, st));
+    int64_t M = 0;
+    if (K > 0) {
+        cub::DoubleBuffer<uint64_t> db(ka.ptr, kb.ptr);
+        FSGC_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, tmp_bytes, db, K, 0, keybits, st));
+        FSGC_CUDA(tmp.alloc(tmp_bytes, st));
+        FSGC_CUDA(cub::DeviceRadixSort::SortKeys(tmp.ptr, tmp_bytes, db, K, 0, keybits, st));
+        uint64_t* sorted = db.Current();
+        uint64_t* other = db.Alternate();
+        size_t ub = 0;
+        FSGC_CUDA(cub::DeviceSelect::Unique(nullptr, ub, sorted, other, dnum.ptr, K, st));
+        if (ub > tmp_bytes) { FSGC_CUDA(tmp.alloc(ub, st)); tmp_bytes = ub; }
+        FSGC_CUDA(cub::DeviceSelect::Unique(tmp.ptr, ub, sorted, other, dnum.ptr, K, st));
+        int64_t nu = 0;
+        uint64_t last = 0;
+        FSGC_CUDA(cudaMemcpyAsync(&nu, dnum.ptr, sizeof nu, cudaMemcpyDeviceToHost, st));
+        FSGC_CUDA(cudaStreamSynchronize(st));
+        if (nu > 0) {
+            FSGC_CUDA(cudaMemcpyAsync(&last, other + nu - 1, sizeof last, cudaMemcpyDeviceToHost, st));
+            FSGC_CUDA(cudaStreamSynchronize(st));
+        }
+        M = (nu > 0 && last == sentinel) ? nu - 1 : nu;
+        if (other != ka.ptr) std::swap(ka.ptr, kb.ptr);  // unique keys now in ka
+    }
+    int bad = 0;
+    FSGC_CUDA(cudaMemcpyAsync(&bad, dbad.ptr, sizeof bad, cudaMemcpyDeviceToHost, st));
+    FSGC_CUDA(cudaStreamSynchronize(st));
+    if (bad) FSGC_FAIL(FSGC_ERR_INVALID, "edge list contains a vertex id outside [0, %lld)", (long long)n);
+    kb.release();
+
+    // 4 degrees of the original ids
+    DevBuf<int64_t> offs_old;
+    FSGC_CUDA(offs_old.alloc(n + 1, st));
+    lower_bounds<<<grid_for(n + 1), 256, 0, st>>>(ka.ptr, M, n, B, offs_old.ptr);
+    FSGC_CUDA(cudaGetLastError());
+
+    // 5 degree order
+    DevBuf<uint64_t> vk, vk2;
+    FSGC_CUDA(vk.alloc(n, st));
+    FSGC_CUDA(vk2.alloc(n, st));
+    degree_keys<<<grid_for(n), 256, 0, st>>>(offs_old.ptr, n, B, vk.ptr);
+    FSGC_CUDA(cudaGetLastError());
+    {
+        int degbits = 1;
+        while ((1ll << degbits) <= M) ++degbits;
+        int endbit = B + degbits;
+        if (endbit > 64) endbit = 64;
+        cub::DoubleBuffer<uint64_t> db(vk.ptr, vk2.ptr);
+        size_t b = 0;
+        FSGC_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, b, db, n, 0, endbit, st));
+        if (b > tmp_bytes) { FSGC_CUDA(tmp.alloc(b, st)); tmp_bytes = b; }
+        FSGC_CUDA(cub::DeviceRadixSort::SortKeys(tmp.ptr, b, db, n, 0, endbit, st));
+        if (db.Current() != vk.ptr) std::swap(vk.ptr, vk2.ptr);
+    }
+    offs_old.release();
+    DevBuf<int32_t> order, rank;
+    DevBuf<int64_t> offs;
+    FSGC_CUDA(order.alloc(n, st));
+    FSGC_CUDA(rank.alloc(n, st));
+    FSGC_CUDA(offs.alloc(n + 1, st));
+    ranks_from_order<<<grid_for(n), 256, 0, st>>>(vk.ptr, n, B, order.ptr, rank.ptr, offs.ptr);
+    FSGC_CUDA(cudaGetLastError());
+    vk.release();
+    vk2.release();
+    {   // offsets = exclusive scan of new-order degrees (in place, n+1 items)
+        FSGC_CUDA(cudaMemsetAsync(offs.ptr + n, 0, sizeof(int64_t), st));
+        size_t b = 0;
+        FSGC_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, b, offs.ptr, offs.ptr, n + 1, st));
+        if (b > tmp_bytes) { FSGC_CUDA(tmp.alloc(b, st)); tmp_bytes = b; }
+        FSGC_CUDA(cub::DeviceScan::ExclusiveSum(tmp.ptr, b, offs.ptr, offs.ptr, n + 1, st));
+    }
+
+    // 6 relabel + sort
+    DevBuf<int32_t> adj, row, osrc, odst;
+    int64_t m = M / 2;
+    if (M > 0) {
+        relabel_keys<<<grid_for(M), 256, 0, st>>>(ka.ptr, M, B, rank.ptr);
+        FSGC_CUDA(cudaGetLastError());
+        FSGC_CUDA(kb.alloc(M, st));
+        cub::DoubleBuffer<uint64_t> db(ka.ptr, kb.ptr);
+        size_t b = 0;
+        FSGC_CUDA(cub::DeviceRadixSort::SortKeys(nullptr, b, db, M, 0, keybits, st));
+        if (b > tmp_bytes) { FSGC_CUDA(tmp.alloc(b, st)); tmp_bytes = b; }
+        FSGC_CUDA(cub::DeviceRadixSort::SortKeys(tmp.ptr, b, db, M, 0, keybits, st));
+        uint64_t* sorted = db.Current();
+        uint64_t* spare = db.Alternate();
+        // 7 CSR arrays + oriented edges
+        FSGC_CUDA(adj.alloc(M, st));
+        FSGC_CUDA(row.alloc(M, st));
+        split_keys<<<grid_for(M), 256, 0, st>>>(sorted, M, B, row.ptr, adj.ptr);
+        FSGC_CUDA(cudaGetLastError());
+        UpperTri pred{B, (1ull << B) - 1};
+        size_t sb = 0;
+        FSGC_CUDA(cub::DeviceSelect::If(nullptr, sb, sorted, spare, dnum.ptr, M, pred, st));
+        if (sb > tmp_bytes) { FSGC_CUDA(tmp.alloc(sb, st)); tmp_bytes = sb; }
+        FSGC_CUDA(cub::DeviceSelect::If(tmp.ptr, sb, sorted, spare, dnum.ptr, M, pred, st));
+        FSGC_CUDA(osrc.alloc(m, st));
+        FSGC_CUDA(odst.alloc(m, st));
+        split_keys<<<grid_for(m), 256, 0, st>>>(spare, m, B, osrc.ptr, odst.ptr);
+        FSGC_CUDA(cudaGetLastError());
+    }
+    tmp.release();
+    ka.release();
+    kb.release();
+    rank.release();
+    int64_t maxdeg = 0;
+    if (n > 0) {
+        int64_t lastoffs[2] = {0, 0};
+        FSGC_CUDA(cudaMemcpyAsync(lastoffs, offs.ptr + n - 1, 2 * sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+        FSGC_CUDA(cudaStreamSynchronize(st));
+        maxdeg = lastoffs[1] - lastoffs[0];  // the last vertex has the largest degree
+    }
+    FSGC_CUDA(cudaStreamSynchronize(st));
+
+    fsgc_graph* g = new fsgc_graph;
+    g->n = n;
+    g->m = m;
+    g->max_degree = maxdeg;
+    g->offsets = offs.take();
+    g->adj = adj.take();
+    g->row = row.take();
+    g->osrc = osrc.take();
+    g->odst = odst.take();
+    g->order = order.take();
+    g->device = dev;
+    *out = g;
+    return FSGC_OK;
+}
+
+extern "C" int fsgc_graph_get_info(const fsgc_graph* g, fsgc_graph_info* o) {
+    if (!g || !o) FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_graph_get_info: null argument");
+    o->num_vertices = g->n;
+    o->num_edges = g->m;
+    o->max_degree = g->max_degree;
+    o->offsets = g->offsets;
+    o->adj = g->adj;
+    o->row = g->row;
+    o->osrc = g->osrc;
+    o->odst = g->odst;
+    o->order = g->order;
+    return FSGC_OK;
+}
+
+extern "C" int fsgc_graph_download(const fsgc_graph* g, int64_t* offsets, int32_t* adj, int32_t* order) {
+    if (!g) FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_graph_download: null graph");
+    if (offsets) FSGC_CUDA(cudaMemcpy(offsets, g->offsets, (g->n + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost));
+    if (adj && g->m > 0) FSGC_CUDA(cudaMemcpy(adj, g->adj, 2 * g->m * sizeof(int32_t), cudaMemcpyDeviceToHost));
+    if (order) FSGC_CUDA(cudaMemcpy(order, g->order, g->n * sizeof(int32_t), cudaMemcpyDeviceToHost));
+    return FSGC_OK;
+}
+
+extern "C" void fsgc_free_graph(fsgc_graph* g) {
+    if (!g) return;
+    cudaFree(g->offsets);
+    cudaFree(g->adj);
+    cudaFree(g->row);
+    cudaFree(g->osrc);
+    cudaFree(g->odst);
+    cudaFree(g->order);
+    delete g;
+}

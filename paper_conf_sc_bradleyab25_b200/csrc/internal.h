@@ -1,0 +1,88 @@
+// internal.h -- shared declarations of the Fringe-SGC library (not public).
+#pragma once
+#include <stdint.h>
+#include <string>
+#include <vector>
+#include <array>
+#include "../../include/fsgc.h"
+
+// --------------------------------------------------------------- errors
+void fsgc_set_error(const char* fmt, ...);
+
+#define FSGC_FAIL(code, ...)            \
+    do {                                \
+        fsgc_set_error(__VA_ARGS__);    \
+        return (code);                  \
+    } while (0)
+
+// --------------------------------------------------------------- handles
+struct fsgc_graph {
+    int64_t n = 0, m = 0, max_degree = 0;
+    int64_t* offsets = nullptr;  // [n+1]
+    int32_t* adj = nullptr;      // [2m]
+    int32_t* row = nullptr;      // [2m]
+    int32_t* osrc = nullptr;     // [m]
+    int32_t* odst = nullptr;     // [m]
+    int32_t* order = nullptr;    // [n]
+    int device = 0;
+};
+
+struct fsgc_pattern {
+    int n = 0;
+    std::vector<std::array<int, 2>> edges;
+    uint64_t adj[FSGC_MAX_PATTERN_VERTICES] = {};
+    uint64_t core_mask = 0;
+    std::vector<int> order;             // matching order (pattern vertex ids)
+    std::vector<uint64_t> type_anchor;  // anchor set per fringe type
+    std::vector<int> type_k;            // fringes per type
+    uint64_t aut = 1, aut_core = 1, aut_core_labeled = 1, fringe_fact = 1;
+};
+
+// --------------------------------------------------------- device program
+// Limits of one count pass (one core-isomorphism class of patterns).
+#define FSGC_MAXC FSGC_MAX_CORE
+#define FSGC_MAXQ FSGC_MAX_VENN_BITS
+#define FSGC_MAXPROG 48
+#define FSGC_MAXT 16
+#define FSGC_MAXPATS FSGC_MAX_BATCH
+#define FSGC_FC_STACK 64
+
+enum { ROOT_ORIENTED = 0, ROOT_DIRECTED = 1, ROOT_VERTEX = 2 };
+
+// A fringe program = one pattern's fringe types seen through one coset
+// representative of the core's automorphisms (anchor sets as Venn bitsets).
+struct FringeProg {
+    uint8_t s;        // number of fringe types
+    uint8_t pat;      // pattern index in the batch
+    uint8_t depth;    // fc stack depth bound
+    uint8_t pad;
+    uint8_t anch[FSGC_MAXT];
+    uint8_t k[FSGC_MAXT];
+};
+
+struct CoreProg {
+    int32_t p;                  // core vertices
+    int32_t q;                  // Venn bits (anchor positions)
+    int32_t nprog;              // fringe programs
+    int32_t npats;              // patterns in the pass
+    int32_t root_mode;          // ROOT_*
+    int32_t pad;
+    uint8_t back[FSGC_MAXC];    // core-adjacency to earlier positions (bitmask)
+    uint8_t gt[FSGC_MAXC];      // symmetry breaking: phi(i) > phi(j) for j in gt[i]
+    int32_t mindeg[FSGC_MAXC];  // degree filter per position
+    int8_t anchor_pos[FSGC_MAXQ];  // Venn bit -> core position
+    int8_t pad2[2];
+    FringeProg prog[FSGC_MAXPROG];
+};
+
+struct PassPlan {
+    CoreProg prog;
+    std::vector<int> members;          // indices into the caller's pattern array
+    std::vector<uint64_t> divisor;     // per member: count = raw / divisor
+    int root_pattern_vertex[FSGC_MAXPATS];
+};
+
+// pattern.cpp
+int fsgc_core_isomorphism(const fsgc_pattern* ref, const fsgc_pattern* other, int* pos_of);
+int fsgc_build_pass(const fsgc_pattern* const* pats, const std::vector<int>& members,
+                    int no_symmetry_breaking, PassPlan* plan);

@@ -1,0 +1,236 @@
+"""GPU parity tests (``-m gpu``): the CUDA path, called through the C ABI,
+against the oracle on the same seeded inputs.  Integer results: bit-exact.
+
+Expected values come only from ``oracle/`` (or the paper, for Fig. 2).
+"""
+import random
+from math import comb
+
+import numpy as np
+import pytest
+
+import oracle
+from inputs import PATTERNS, fig2_edges, workload_edges, rmat_edges_np
+from inputs.patterns import all_connected_patterns, star
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():  # pragma: no cover
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+import paper_conf_sc_bradleyab25_b200 as F  # noqa: E402
+
+
+def oracle_graph(n, edges):
+    offs, adj, order = oracle.degree_ordered_csr(n, edges)
+    return offs, adj, order, oracle.csr_to_adjacency(offs, adj)
+
+
+def count_all(g, pats, **kw):
+    out = []
+    for i in range(0, len(pats), 16):
+        out += F.fsgc_count(g, pats[i:i + 16], **kw)
+    return out
+
+
+_cache = {}
+
+
+def workload(name):
+    if name not in _cache:
+        n, e = workload_edges(name)
+        _cache[name] = (n, e, oracle_graph(n, e))
+    return _cache[name]
+
+
+# ------------------------------------------------------------ graph loading
+
+def _rand_multigraph(n, E, seed):
+    rng = np.random.default_rng(seed)
+    return rng.integers(0, n, size=(E, 2))
+
+
+@pytest.mark.parametrize("case", ["fig2", "pl2k", "multi", "rmat10", "isolated", "empty", "int32", "device"])
+def test_load_graph_bit_exact(case):
+    if case == "fig2":
+        n, e = fig2_edges()
+    elif case == "pl2k":
+        n, e, _ = workload("pl2k")
+    elif case == "multi":
+        n, e = 300, _rand_multigraph(300, 5000, 1)          # duplicates + loops
+    elif case == "rmat10":
+        n, e = 1 << 10, rmat_edges_np(10, 8, seed=2)
+    elif case == "isolated":
+        n, e = 1000, _rand_multigraph(50, 400, 3)           # vertices 50..999 isolated
+    elif case == "empty":
+        n, e = 7, np.zeros((0, 2), dtype=np.int64)
+    elif case == "int32":
+        n, e = 500, _rand_multigraph(500, 3000, 4).astype(np.int32)
+    else:
+        n, e = 800, _rand_multigraph(800, 6000, 5)
+    src = torch.from_numpy(np.ascontiguousarray(e)).cuda() if case == "device" else e
+    g = F.fsgc_load_graph(src, n)
+    offs, adj, order = g.download()
+    eo, ea, eord = oracle.degree_ordered_csr(n, e)
+    assert np.array_equal(offs, eo)
+    assert np.array_equal(adj, ea)
+    assert np.array_equal(order, eord)
+    assert g.m == len(ea) // 2
+    assert g.max_degree == (int(np.diff(eo).max()) if n else 0)
+
+
+def test_load_graph_rejects_bad_ids():
+    with pytest.raises(F.FsgcError):
+        F.fsgc_load_graph(np.array([[0, 1], [1, 5]]), 5)
+    with pytest.raises(F.FsgcError):
+        F.fsgc_load_graph(np.array([[0, -1]]), 5)
+
+
+# ------------------------------------------------------------ counts
+
+def test_fig2_paper_values():
+    """Sec. 1: 1 triangle, 5 tailed triangles; Sec. 3: 35 3-stars."""
+    n, e = fig2_edges()
+    g = F.fsgc_load_graph(e, n)
+    pats = [F.compile_named(PATTERNS[x]) for x in ("triangle", "1-tailed-triangle", "3-star")]
+    res = F.fsgc_count(g, pats)
+    assert [r.count for r in res] == [1, 5, 35]
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_all_small_patterns_random_graphs(seed):
+    """All 31 connected patterns <= 5 vertices on random graphs vs mode-1
+    brute force (Sec. 3.4's exhaustive check, on the GPU path)."""
+    rng = random.Random(seed)
+    n = 12 + 3 * seed
+    edges = [(a, b) for a in range(n) for b in range(a + 1, n) if rng.random() < 0.35]
+    g = F.fsgc_load_graph(np.array(edges, dtype=np.int64).reshape(-1, 2), n)
+    _, _, _, gadj = oracle_graph(n, edges)
+    pats = all_connected_patterns(5)
+    res = count_all(g, [F.compile_named(P) for P in pats])
+    for P, r in zip(pats, res):
+        assert not r.overflow
+        assert r.count == oracle.brute_force_count(gadj, P.n, P.edges), P
+
+
+PL2K_PATTERNS = ["1-tailed-triangle", "2-tailed-triangle", "3-tailed-triangle", "4-tailed-triangle",
+                 "triangle", "wedge", "3-star", "6-star", "path4", "path5", "cycle4", "clique4",
+                 "diamond", "fig4", "k4core+2f", "k4core+6f", "diamondcore+3f", "tricore+4f",
+                 "tricore+6f", "c4core+2f", "clique5", "cycle5"]
+
+
+def test_pl2k_named_patterns():
+    """configs[0] graph (2,000 vertices / 10,000 edges) -- every named pattern
+    vs the oracle's core+fringe mode (itself pinned to brute force)."""
+    n, e, (_, _, _, gadj) = workload("pl2k")
+    g = F.fsgc_load_graph(e, n)
+    pats = [PATTERNS[x] for x in PL2K_PATTERNS]
+    res = count_all(g, [F.compile_named(P) for P in pats])
+    for P, r in zip(pats, res):
+        want = oracle.fringe_count(gadj, P.n, P.edges, P.core)
+        assert not r.overflow and r.count == want, (P.name, r.count, want)
+
+
+def test_symmetry_breaking_invariant():
+    """sum over symmetry-broken core instances x fringe programs == sum over
+    all injective core maps (divided consistently)."""
+    n, e, _ = workload("pl2k")
+    g = F.fsgc_load_graph(e, n)
+    pats = [F.compile_named(PATTERNS[x]) for x in ["1-tailed-triangle", "cycle4", "clique4", "diamond",
+                                                     "fig4", "k4core+3f", "diamondcore+2f", "c4core+4f"]]
+    a = count_all(g, pats)
+    b = count_all(g, pats, no_symmetry_breaking=True)
+    for x, y in zip(a, b):
+        assert x.count == y.count and x.count is not None
+
+
+def test_batch_equals_single_and_shards_partition():
+    n, e, _ = workload("internet")
+    g = F.fsgc_load_graph(e, n)
+    pats = [F.compile_named(PATTERNS[f"{k}-tailed-triangle"]) for k in range(1, 5)]
+    batch = F.fsgc_count(g, pats)
+    for p, r in zip(pats, batch):
+        assert F.fsgc_count(g, [p])[0].count == r.count
+    for shards in (2, 3, 8):
+        raws = [0] * 4
+        for s in range(shards):
+            part = F.fsgc_count(g, pats, shard_index=s, shard_count=shards)
+            for k in range(4):
+                raws[k] += part[k].raw
+        assert raws == [r.raw for r in batch]
+
+
+def test_internet_full_size_bench_config():
+    """configs[1] at full size, in the launch configuration bench.py times
+    (one batched pass over the 4 k-tailed triangles): every count exact."""
+    n, e, (_, _, _, gadj) = workload("internet")
+    g = F.fsgc_load_graph(e, n)
+    pats = [PATTERNS[f"{k}-tailed-triangle"] for k in range(1, 5)]
+    res = F.fsgc_count(g, [F.compile_named(P) for P in pats])
+    for P, r in zip(pats, res):
+        assert r.count == oracle.fringe_count(gadj, P.n, P.edges), P.name
+
+
+@pytest.mark.parametrize("wl", ["internet", "rmat16"])
+def test_sampled_roots_no_symmetry(wl):
+    """Per-root-vertex raw sums (no symmetry breaking) for sampled roots,
+    low and high degree, vs oracle.root_raw_sum."""
+    n, e, (offs, _, _, gadj) = workload(wl)
+    g = F.fsgc_load_graph(e, n)
+    rng = random.Random(3)
+    deg = np.diff(offs)
+    if wl == "internet":   # d_max ~170: the hubs themselves are cheap for the oracle
+        cands = [n - 1 - i for i in range(5)] + rng.sample(range(n), 10)
+    else:                  # RMAT hubs are too heavy for a per-root Python oracle
+        ok = [v for v in range(n) if 1 <= deg[v] <= 48]
+        cands = rng.sample(ok, 10) + [ok[-1]]
+    names = ["1-tailed-triangle", "4-tailed-triangle", "diamond", "tricore+3f"] if wl == "internet" \
+        else ["1-tailed-triangle", "cycle4", "diamond", "k4core+2f"]
+    for name in names:
+        P = PATTERNS[name]
+        p = F.compile_named(P)
+        for r in cands:
+            if p.info.core_size == 1:
+                b, e_ = r, r + 1
+            else:
+                b, e_ = int(offs[r]), int(offs[r + 1])
+            res = F.fsgc_count(g, [p], root_begin=b, root_end=e_, no_symmetry_breaking=True)[0]
+            want = oracle.root_raw_sum(gadj, P.n, P.edges, P.core, res.root_pattern_vertex, r)
+            assert res.raw == want, (name, r, res.raw, want)
+
+
+def test_overflow_and_192bit_binomials():
+    """Star graph with 200,000 leaves: C(200000, 8) < 2^128 but 8*C(n,8) >
+    2^128 (exercises the 192-bit intermediate); C(200000, 9) > 2^128 must be
+    flagged, never wrapped."""
+    L = 200000
+    e = np.stack([np.zeros(L, dtype=np.int64), np.arange(1, L + 1)], axis=1)
+    g = F.fsgc_load_graph(e, L + 1)
+    r7, r8, r9 = F.fsgc_count(g, [F.compile_named(star(k)) for k in (7, 8, 9)])
+    assert r7.count == comb(L, 7) and r8.count == comb(L, 8)
+    assert comb(L, 8) < 1 << 128 < 8 * comb(L, 8)
+    assert r9.overflow and r9.count is None and comb(L, 9) >= 1 << 128
+
+
+def test_degenerate_inputs():
+    g = F.fsgc_load_graph(np.zeros((0, 2), dtype=np.int64), 5)
+    res = F.fsgc_count(g, [F.compile_named(PATTERNS[x]) for x in ("vertex", "edge", "triangle", "3-star")])
+    assert [r.count for r in res] == [5, 0, 0, 0]
+    n, e = fig2_edges()
+    g = F.fsgc_load_graph(e, n)
+    big = F.compile_named(PATTERNS["clique5"])
+    assert F.fsgc_count(g, [big])[0].count == 0
+    r = F.fsgc_count(g, [F.compile_named(PATTERNS["edge"])], root_begin=3, root_end=3)[0]
+    assert r.raw == 0
+    assert F.fsgc_count(g, [F.compile_named(PATTERNS["vertex"]), F.compile_named(PATTERNS["edge"])]) [1].count == 8
+
+
+def test_degree_filter_off_counts_core_instances():
+    n, e, (_, _, _, gadj) = workload("pl2k")
+    g = F.fsgc_load_graph(e, n)
+    for name in ["1-tailed-triangle", "clique4", "cycle4"]:
+        P = PATTERNS[name]
+        r = F.fsgc_count(g, [F.compile_named(P)], no_degree_filter=True)[0]
+        assert r.core_matches == oracle.core_matches(gadj, P.n, P.edges, P.core), name
+        assert r.count == F.fsgc_count(g, [F.compile_named(P)])[0].count
