@@ -160,11 +160,11 @@ __device__ __forceinline__ void atomic_add_u128(AccDev* a, u128 v, bool ovf) {
 }
 
 // per-warp epilogue: reduce the lane accumulators, one atomic per pattern
-__device__ __forceinline__ void warp_flush_acc(int npats, u128* acc_l, bool ovf, unsigned long long nmatch,
+__device__ __forceinline__ void warp_flush_acc(int npats, u128* acc_l, uint32_t ovf_mask, unsigned long long nmatch,
                                                AccDev* acc, unsigned long long* matches, int lane) {
     for (int pi = 0; pi < npats; ++pi) {
         u128 v = acc_l[pi];
-        bool o = ovf;
+        bool o = (ovf_mask >> pi) & 1;
         warp_reduce_u128(v, o);
         if (lane == 0 && (v != 0 || o)) atomic_add_u128(acc + pi, v, o);
     }
@@ -181,7 +181,7 @@ __global__ void __launch_bounds__(256) vertex_core_kernel(GraphDev G, const Core
     const int lane = threadIdx.x & 31;
     u128 acc_l[FSGC_MAXPATS];
     for (int i = 0; i < FSGC_MAXPATS; ++i) acc_l[i] = 0;
-    bool ovf = false;
+    uint32_t ovf_mask = 0;   // per-pattern overflow bits
     unsigned long long nmatch = 0;
     const int64_t total = W.end - W.begin;
     const int64_t nchunks = (total + W.chunk - 1) / W.chunk;
@@ -200,11 +200,13 @@ __global__ void __launch_bounds__(256) vertex_core_kernel(GraphDev G, const Core
         uint32_t venn[2] = {0, deg};
         for (int pi = 0; pi < P.nprog; ++pi) {
             const FringeProg fp = P.prog[pi];
-            u128 c2 = fc_eval(venn, P.q, fp, ovf);
-            acc_l[fp.pat] = add_ovf(acc_l[fp.pat], c2, ovf);
+            bool o = false;
+            u128 c2 = fc_eval(venn, P.q, fp, o);
+            acc_l[fp.pat] = add_ovf(acc_l[fp.pat], c2, o);
+            if (o) ovf_mask |= 1u << fp.pat;
         }
     }
-    warp_flush_acc(P.npats, acc_l, ovf, nmatch, acc, matches, lane);
+    warp_flush_acc(P.npats, acc_l, ovf_mask, nmatch, acc, matches, lane);
 }
 
 // ------------------------------------------------------------------------
@@ -221,7 +223,7 @@ __global__ void __launch_bounds__(WARPS * 32) core_kernel(GraphDev G, const Core
     int nbuf = 0;
     u128 acc_l[FSGC_MAXPATS];
     for (int i = 0; i < FSGC_MAXPATS; ++i) acc_l[i] = 0;
-    bool ovf = false;
+    uint32_t ovf_mask = 0;   // per-pattern overflow bits
     unsigned long long nmatch = 0;
 
     int emb[FSGC_MAXC];
@@ -240,8 +242,10 @@ __global__ void __launch_bounds__(WARPS * 32) core_kernel(GraphDev G, const Core
             uint32_t vloc[1 << FSGC_MAXQ];
             for (int e = 0; e < V; ++e) vloc[e] = vbuf[vi * V + e];
             const FringeProg fp = P.prog[pi];
-            u128 c = fc_eval(vloc, q, fp, ovf);
-            acc_l[fp.pat] = add_ovf(acc_l[fp.pat], c, ovf);
+            bool o = false;
+            u128 c = fc_eval(vloc, q, fp, o);
+            acc_l[fp.pat] = add_ovf(acc_l[fp.pat], c, o);
+            if (o) ovf_mask |= 1u << fp.pat;
         }
         nbuf = 0;
         __syncwarp();
@@ -373,7 +377,7 @@ __global__ void __launch_bounds__(WARPS * 32) core_kernel(GraphDev G, const Core
         }
     }
     if (nbuf) flush();
-    warp_flush_acc(P.npats, acc_l, ovf, nmatch, acc, matches, lane);
+    warp_flush_acc(P.npats, acc_l, ovf_mask, nmatch, acc, matches, lane);
 }
 
 int sm_count() {
@@ -449,8 +453,25 @@ extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, 
     cudaStream_t st = (cudaStream_t)stream_;
     std::memset(results, 0, sizeof(fsgc_result) * npats);
 
-    auto groups = group_patterns(pats, npats);
-    for (auto& members : groups) {
+    // passes: isomorphic cores share one pass (one Venn per core match for
+    // all their fringe programs) as long as the pass fits the program limits
+    std::vector<std::vector<int>> passes;
+    for (auto& grp : group_patterns(pats, npats)) {
+        std::vector<int> cur;
+        for (int idx : grp) {
+            std::vector<int> trial = cur;
+            trial.push_back(idx);
+            PassPlan probe;
+            if (!cur.empty() && fsgc_build_pass(pats, trial, opts.no_symmetry_breaking, &probe) != FSGC_OK) {
+                passes.push_back(cur);
+                cur = {idx};
+            } else {
+                cur = trial;
+            }
+        }
+        if (!cur.empty()) passes.push_back(cur);
+    }
+    for (auto& members : passes) {
         PassPlan plan;
         int rc = fsgc_build_pass(pats, members, opts.no_symmetry_breaking, &plan);
         if (rc) return rc;
