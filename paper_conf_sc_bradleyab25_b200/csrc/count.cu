@@ -22,8 +22,11 @@
 // chunks round-robin across GPUs.
 #include <algorithm>
 #include <cstring>
+#include <map>
+#include <mutex>
 #include "devbuf.cuh"
 #include "u128.cuh"
+#include "fc.cuh"
 
 #define FULLMASK 0xffffffffu
 
@@ -67,68 +70,6 @@ __device__ __forceinline__ int upper_bound(const int32_t* __restrict__ L, int le
         if (__ldg(L + mid) <= x) lo = mid + 1; else hi = mid;
     }
     return lo;
-}
-
-struct Frame {
-    u128 M;
-    uint32_t vc;
-    uint8_t pos, rem, idx, i, top, kind;
-};
-
-// Iterative Listing 5: the recursion fc(pos, rem, idx) with an explicit
-// stack.  `venn` is this lane's private copy; it is decremented/restored
-// exactly as lines 10/12 and 18/20 of the listing do.
-__device__ u128 fc_eval(uint32_t* venn, int q, const FringeProg& P, bool& ovf) {
-    const int s = P.s;
-    if (s == 0) return 1;
-    const int full = (1 << q) - 1;
-    Frame st[FSGC_FC_STACK];
-    int sp = 0;
-    u128 total = 0;
-    int pos = 0, rem = P.k[0], idx = P.anch[0];
-    u128 M = 1;
-    for (;;) {
-        // ---- enter fc(pos, rem, idx) with multiplier M
-        for (;;) {
-            if (rem == 0) {                              // line 6: next type
-                if (++pos == s) { total = add_ovf(total, M, ovf); break; }  // line 5
-                rem = P.k[pos];
-                idx = P.anch[pos];
-                continue;
-            }
-            const uint32_t vc = venn[idx];               // line 7
-            if (idx == full) {                           // line 8: last entry
-                if ((uint32_t)rem > vc) break;           // line 9: no solution
-                M = mul_ovf(M, binom_ovf(vc, (uint32_t)rem, ovf), ovf);  // line 11
-                venn[idx] = vc - rem;                    // line 10
-                Frame f;
-                f.kind = 0; f.idx = (uint8_t)idx; f.rem = (uint8_t)rem;
-                st[sp++] = f;
-                rem = 0;
-                continue;
-            }
-            const int top = min(rem, (int)vc);           // line 16
-            Frame f;
-            f.M = M; f.vc = vc; f.pos = (uint8_t)pos; f.rem = (uint8_t)rem;
-            f.idx = (uint8_t)idx; f.i = 0; f.top = (uint8_t)top; f.kind = 1;
-            st[sp++] = f;                                 // i = 0: C(vc,0) = 1
-            idx = (idx + 1) | P.anch[pos];               // line 19: next entry
-        }
-        // ---- return: undo and advance the innermost open summation
-        for (;;) {
-            if (sp == 0) return total;
-            Frame& f = st[sp - 1];
-            if (f.kind == 0) { venn[f.idx] += f.rem; --sp; continue; }  // line 12
-            venn[f.idx] += f.i;                          // line 20
-            if (++f.i > f.top) { --sp; continue; }
-            venn[f.idx] -= f.i;                          // line 18
-            M = mul_ovf(f.M, binom_ovf(f.vc, f.i, ovf), ovf);
-            pos = f.pos;
-            rem = f.rem - f.i;
-            idx = (f.idx + 1) | P.anch[f.pos];
-            break;
-        }
-    }
 }
 
 __device__ __forceinline__ void warp_reduce_u128(u128& v, bool& ovf) {
@@ -201,9 +142,136 @@ __global__ void __launch_bounds__(256) vertex_core_kernel(GraphDev G, const Core
         for (int pi = 0; pi < P.nprog; ++pi) {
             const FringeProg fp = P.prog[pi];
             bool o = false;
-            u128 c2 = fc_eval(venn, P.q, fp, o);
+            u128 c2 = fc_dispatch<4>(venn, P.q, fp, o);
             acc_l[fp.pat] = add_ovf(acc_l[fp.pat], c2, o);
             if (o) ovf_mask |= 1u << fp.pat;
+        }
+    }
+    warp_flush_acc(P.npats, acc_l, ovf_mask, nmatch, acc, matches, lane);
+}
+
+// ------------------------------------------------------------------------
+// 2-vertex (edge) cores: ONE LANE PER ROOT EDGE.  The Venn diagram of an edge
+// core is {|e(u)\e(v)|, |e(v)\e(u)|, |e(u)&e(v)|} = {du-1-c, dv-1-c, c} with
+// c = |N(u) & N(v)| (u, v are not in N(u) & N(v); v in N(u)).  A lane merges
+// (or gallops through) the two sorted lists itself when the shorter list has
+// <= HEAVY entries; heavier roots are ballot-collected and processed by the
+// whole warp one after another (Listing 7's "all lanes process the first such
+// vertex together"), lanes over the shorter list binary-searching the longer.
+// fc is Sec. 3.1's closed form (the paper's specialised 2-core code).
+constexpr int kHeavy = 32;
+
+__device__ __forceinline__ int intersect_seq(const int32_t* __restrict__ A, int na, const int32_t* __restrict__ B,
+                                             int nb) {
+    if (na > nb) { const int32_t* t = A; A = B; B = t; int x = na; na = nb; nb = x; }
+    int c = 0;
+    if (na == 0) return 0;
+    if (nb > 8 * na) {                      // galloping search of A's elements in B
+        int j = 0;
+        for (int i = 0; i < na && j < nb; ++i) {
+            const int x = __ldg(A + i);
+            int step = 1, hi = j;
+            while (hi < nb && __ldg(B + hi) < x) { j = hi + 1; hi += step; step <<= 1; }
+            if (hi > nb) hi = nb;
+            int lo = j;                      // B[lo-1] < x, search [lo, hi]
+            int h2 = hi;
+            while (lo < h2) {
+                int mid = (lo + h2) >> 1;
+                if (__ldg(B + mid) < x) lo = mid + 1; else h2 = mid;
+            }
+            j = lo;
+            if (j < nb && __ldg(B + j) == x) { ++c; ++j; }
+        }
+        return c;
+    }
+    int i = 0, j = 0;                        // linear merge
+    int a = __ldg(A), b = __ldg(B);
+    for (;;) {
+        if (a < b) { if (++i == na) break; a = __ldg(A + i); }
+        else if (a > b) { if (++j == nb) break; b = __ldg(B + j); }
+        else {
+            ++c;
+            if (++i == na || ++j == nb) break;
+            a = __ldg(A + i);
+            b = __ldg(B + j);
+        }
+    }
+    return c;
+}
+
+// whole warp: |A & B|, lanes over the shorter list, binary search in the longer
+__device__ __forceinline__ int intersect_warp(const int32_t* __restrict__ A, int na, const int32_t* __restrict__ B,
+                                              int nb, int lane) {
+    if (na > nb) { const int32_t* t = A; A = B; B = t; int x = na; na = nb; nb = x; }
+    int c = 0;
+    for (int b0 = 0; b0 < na; b0 += 32) {
+        const int i = b0 + lane;
+        bool hit = false;
+        if (i < na) hit = contains(B, nb, __ldg(A + i));
+        c += __popc(__ballot_sync(FULLMASK, hit));
+    }
+    return c;
+}
+
+template <class A>
+__device__ __forceinline__ void edge_programs(const CoreProg& P, uint64_t nu, uint64_t nv, uint64_t nuv,
+                                              u128* acc_l, uint32_t& ovf_mask) {
+    for (int pi = 0; pi < P.nprog; ++pi) {
+        bool o = false;
+        const int pat = P.prog[pi].pat;
+        u128 c = A::widen(edge_formula<A>(nu, nv, nuv, P.ek[pi], P.el[pi], P.em[pi], o));
+        acc_l[pat] = add_ovf(acc_l[pat], c, o);
+        if (o) ovf_mask |= 1u << pat;
+    }
+}
+
+__global__ void __launch_bounds__(256) edge_core_kernel(GraphDev G, const CoreProg P, WorkDesc W, AccDev* acc,
+                                                        unsigned long long* matches, unsigned long long* queue) {
+    const int lane = threadIdx.x & 31;
+    u128 acc_l[FSGC_MAXPATS];
+    for (int i = 0; i < FSGC_MAXPATS; ++i) acc_l[i] = 0;
+    uint32_t ovf_mask = 0;
+    unsigned long long nmatch = 0;
+    int Kmax = 0;
+    for (int pi = 0; pi < P.nprog; ++pi) Kmax = max(Kmax, (int)P.prog[pi].ksum);
+    const int64_t total = W.end - W.begin;
+    for (;;) {
+        unsigned long long jq = 0;
+        if (lane == 0) jq = atomicAdd(queue, 1ull);
+        jq = __shfl_sync(FULLMASK, jq, 0);
+        const int64_t g = (int64_t)jq * W.nshards + W.shard;
+        const int64_t t0 = g * 32;
+        if (t0 >= total) break;
+        const int64_t t = t0 + lane;
+        bool active = t < total;
+        int u = 0, v = 0;
+        int64_t ou = 0, ov = 0;
+        int du = 0, dv = 0;
+        if (active) {
+            const int64_t item = W.end - 1 - t;          // heavy roots first
+            if (P.root_mode == ROOT_ORIENTED) { u = __ldg(G.osrc + item); v = __ldg(G.odst + item); }
+            else { u = __ldg(G.row + item); v = __ldg(G.adj + item); }
+            ou = __ldg(G.offs + u); du = (int)(__ldg(G.offs + u + 1) - ou);
+            ov = __ldg(G.offs + v); dv = (int)(__ldg(G.offs + v + 1) - ov);
+            if (W.degfilter && (du < P.mindeg[0] || dv < P.mindeg[1])) active = false;
+        }
+        const bool heavy = active && min(du, dv) > kHeavy;
+        int c = 0;
+        if (active && !heavy) c = intersect_seq(G.adj + ou, du, G.adj + ov, dv);
+        unsigned hb = __ballot_sync(FULLMASK, heavy);
+        while (hb) {
+            const int who = __ffs(hb) - 1;
+            hb &= hb - 1;
+            const int64_t wou = __shfl_sync(FULLMASK, ou, who), wov = __shfl_sync(FULLMASK, ov, who);
+            const int wdu = __shfl_sync(FULLMASK, du, who), wdv = __shfl_sync(FULLMASK, dv, who);
+            const int cc = intersect_warp(G.adj + wou, wdu, G.adj + wov, wdv, lane);
+            if (lane == who) c = cc;
+        }
+        if (active) {
+            ++nmatch;
+            const uint64_t nu = du - 1 - c, nv = dv - 1 - c, nuv = c;
+            if (fits64(nu + nv + nuv, Kmax)) edge_programs<Exact64>(P, nu, nv, nuv, acc_l, ovf_mask);
+            else edge_programs<Checked128>(P, nu, nv, nuv, acc_l, ovf_mask);
         }
     }
     warp_flush_acc(P.npats, acc_l, ovf_mask, nmatch, acc, matches, lane);
@@ -243,7 +311,7 @@ __global__ void __launch_bounds__(WARPS * 32) core_kernel(GraphDev G, const Core
             for (int e = 0; e < V; ++e) vloc[e] = vbuf[vi * V + e];
             const FringeProg fp = P.prog[pi];
             bool o = false;
-            u128 c = fc_eval(vloc, q, fp, o);
+            u128 c = fc_dispatch<FSGC_FC_STACK>(vloc, q, fp, o);
             acc_l[fp.pat] = add_ovf(acc_l[fp.pat], c, o);
             if (o) ovf_mask |= 1u << fp.pat;
         }
@@ -454,27 +522,49 @@ extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, 
     std::memset(results, 0, sizeof(fsgc_result) * npats);
 
     // passes: isomorphic cores share one pass (one Venn per core match for
-    // all their fringe programs) as long as the pass fits the program limits
-    std::vector<std::vector<int>> passes;
-    for (auto& grp : group_patterns(pats, npats)) {
-        std::vector<int> cur;
-        for (int idx : grp) {
-            std::vector<int> trial = cur;
-            trial.push_back(idx);
-            PassPlan probe;
-            if (!cur.empty() && fsgc_build_pass(pats, trial, opts.no_symmetry_breaking, &probe) != FSGC_OK) {
-                passes.push_back(cur);
-                cur = {idx};
-            } else {
-                cur = trial;
+    // all their fringe programs) as long as the pass fits the program limits.
+    // Plans depend only on the patterns and the mode: cached by pattern uid.
+    std::vector<uint64_t> key;
+    for (int i = 0; i < npats; ++i) key.push_back(pats[i]->uid);
+    key.push_back(opts.no_symmetry_breaking ? 1 : 0);
+    std::vector<PassPlan> plans;
+    {
+        static std::mutex mu;
+        static std::map<std::vector<uint64_t>, std::vector<PassPlan>> cache;
+        std::lock_guard<std::mutex> lock(mu);
+        auto it = cache.find(key);
+        if (it != cache.end()) {
+            plans = it->second;
+        } else {
+            std::vector<std::vector<int>> passes;
+            for (auto& grp : group_patterns(pats, npats)) {
+                std::vector<int> cur;
+                for (int idx : grp) {
+                    std::vector<int> trial = cur;
+                    trial.push_back(idx);
+                    PassPlan probe;
+                    if (!cur.empty() && fsgc_build_pass(pats, trial, opts.no_symmetry_breaking, &probe) != FSGC_OK) {
+                        passes.push_back(cur);
+                        cur = {idx};
+                    } else {
+                        cur = trial;
+                    }
+                }
+                if (!cur.empty()) passes.push_back(cur);
             }
+            for (auto& members : passes) {
+                PassPlan plan;
+                int rc = fsgc_build_pass(pats, members, opts.no_symmetry_breaking, &plan);
+                if (rc) return rc;
+                plans.push_back(plan);
+            }
+            if (cache.size() > 1024) cache.clear();
+            cache[key] = plans;
         }
-        if (!cur.empty()) passes.push_back(cur);
     }
-    for (auto& members : passes) {
-        PassPlan plan;
-        int rc = fsgc_build_pass(pats, members, opts.no_symmetry_breaking, &plan);
-        if (rc) return rc;
+    for (const PassPlan& plan : plans) {
+        const std::vector<int>& members = plan.members;
+        int rc = FSGC_OK;
         const CoreProg& cp = plan.prog;
         const int64_t R = roots_for(g, cp.root_mode);
         int64_t b = opts.root_begin < 0 ? 0 : opts.root_begin;
@@ -509,6 +599,17 @@ extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, 
                 grid = std::max<int64_t>(1, std::min<int64_t>(grid, (int64_t)sm_count() * 8));
                 vertex_core_kernel<<<(int)grid, 256, 0, st>>>(G, cp, W, dacc, dmatch);
                 FSGC_CUDA(cudaGetLastError());
+            } else if (cp.p == 2) {
+                int per_sm = 0;
+                FSGC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, edge_core_kernel, 256, 0));
+                if (per_sm < 1) per_sm = 1;
+                W.chunk = 32;
+                int64_t nchunks = ((e - b) + 31) / 32;
+                int64_t mine = (nchunks + opts.shard_count - 1) / opts.shard_count;
+                int64_t grid = std::min<int64_t>((int64_t)sm_count() * per_sm, (mine + 7) / 8);
+                if (grid < 1) grid = 1;
+                edge_core_kernel<<<(int)grid, 256, 0, st>>>(G, cp, W, dacc, dmatch, dqueue);
+                FSGC_CUDA(cudaGetLastError());
             } else {
                 const size_t smem = (size_t)kWarps * 33 * (1u << cp.q) * sizeof(uint32_t);
                 static bool attr_set = false;
@@ -529,10 +630,11 @@ extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, 
             }
         }
         FSGC_CUDA(cudaEventRecord(ev1, st));
-        AccDev hacc[FSGC_MAXPATS];
-        unsigned long long hmatch = 0;
-        FSGC_CUDA(cudaMemcpyAsync(hacc, dacc, acc_bytes, cudaMemcpyDeviceToHost, st));
-        FSGC_CUDA(cudaMemcpyAsync(&hmatch, dmatch, sizeof hmatch, cudaMemcpyDeviceToHost, st));
+        struct { AccDev acc[FSGC_MAXPATS]; unsigned long long match; } host;
+        static_assert(sizeof(host) == sizeof(AccDev) * FSGC_MAXPATS + 8, "layout");
+        FSGC_CUDA(cudaMemcpyAsync(&host, dacc, sizeof host, cudaMemcpyDeviceToHost, st));
+        const AccDev* hacc = host.acc;
+        const unsigned long long hmatch = host.match;
         FSGC_CUDA(cudaStreamSynchronize(st));
         float kms = 0.f;
         FSGC_CUDA(cudaEventElapsedTime(&kms, ev0, ev1));

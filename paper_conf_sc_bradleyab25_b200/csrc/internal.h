@@ -28,6 +28,7 @@ struct fsgc_graph {
 };
 
 struct fsgc_pattern {
+    uint64_t uid = 0;                   // unique per compiled pattern (plan cache key)
     int n = 0;
     std::vector<std::array<int, 2>> edges;
     uint64_t adj[FSGC_MAX_PATTERN_VERTICES] = {};
@@ -55,7 +56,7 @@ struct FringeProg {
     uint8_t s;        // number of fringe types
     uint8_t pat;      // pattern index in the batch
     uint8_t depth;    // fc stack depth bound
-    uint8_t pad;
+    uint8_t ksum;     // total fringes (sum of k) -- for the 64-bit bound
     uint8_t anch[FSGC_MAXT];
     uint8_t k[FSGC_MAXT];
 };
@@ -73,6 +74,9 @@ struct CoreProg {
     int8_t anchor_pos[FSGC_MAXQ];  // Venn bit -> core position
     int8_t pad2[2];
     FringeProg prog[FSGC_MAXPROG];
+    // edge cores (p == 2): each program as (k tails on c0, l tails on c1,
+    // m wedge fringes on {c0,c1}) for the Sec. 3.1 closed form
+    uint8_t ek[FSGC_MAXPROG], el[FSGC_MAXPROG], em[FSGC_MAXPROG];
 };
 
 struct PassPlan {

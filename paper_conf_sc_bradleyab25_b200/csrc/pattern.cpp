@@ -10,6 +10,7 @@
 #include "internal.h"
 
 #include <algorithm>
+#include <atomic>
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
@@ -266,6 +267,8 @@ extern "C" int fsgc_compile_pattern(int n, const int32_t* edges, int ne, const i
         std::sort(img.begin(), img.end());
         if (img == tpos) P.aut_core_labeled++;
     }
+    static std::atomic<uint64_t> next_uid{1};
+    P.uid = next_uid.fetch_add(1);
     *out = new fsgc_pattern(P);
     return FSGC_OK;
 }
@@ -419,20 +422,35 @@ int fsgc_build_pass(const fsgc_pattern* const* pats, const std::vector<int>& mem
         fp.pat = (uint8_t)progs[k].pat;
         if (progs[k].types.size() > FSGC_MAXT) FSGC_FAIL(FSGC_ERR_PATTERN, "too many fringe types");
         fp.s = (uint8_t)progs[k].types.size();
-        int depth = 0;
+        int depth = 0, ksum = 0;
         int att[FSGC_MAXC] = {};
-        for (size_t t = 0; t < progs[k].types.size(); ++t) {
-            uint64_t m = progs[k].types[t].first;
-            int kk = progs[k].types[t].second;
+        // fc is independent of the fringe-type order (Sec. 3.2 "we can start
+        // with any fringe type"); most constrained (largest anchor set) first
+        // makes infeasible programs fail at the first, smallest Venn entries
+        std::vector<std::pair<uint64_t, int>> ts = progs[k].types;
+        std::stable_sort(ts.begin(), ts.end(), [](const std::pair<uint64_t, int>& a, const std::pair<uint64_t, int>& b) {
+            return popc64(a.first) > popc64(b.first);
+        });
+        for (size_t t = 0; t < ts.size(); ++t) {
+            uint64_t m = ts[t].first;
+            int kk = ts[t].second;
             if (kk > 255) FSGC_FAIL(FSGC_ERR_PATTERN, "more than 255 fringes of one type");
             uint8_t vb = 0;
             for (uint64_t a = m; a; a &= a - 1) { vb |= (uint8_t)(1u << bit_of[ctz64(a)]); att[ctz64(a)] += kk; }
             fp.anch[t] = vb;
             fp.k[t] = (uint8_t)kk;
             depth += 1 << (cp.q - popc64(vb));
+            ksum += kk;
+            if (p == 2) {
+                if (m == 1) cp.ek[k] = (uint8_t)kk;
+                else if (m == 2) cp.el[k] = (uint8_t)kk;
+                else cp.em[k] = (uint8_t)kk;
+            }
         }
         if (depth > FSGC_FC_STACK) FSGC_FAIL(FSGC_ERR_PATTERN, "fringe program too deep (%d)", depth);
+        if (ksum > 255) FSGC_FAIL(FSGC_ERR_PATTERN, "more than 255 fringes");
         fp.depth = (uint8_t)depth;
+        fp.ksum = (uint8_t)ksum;
         for (int i = 0; i < p; ++i) cp.mindeg[i] = std::min(cp.mindeg[i], att[i]);
     }
     for (int i = 0; i < p; ++i) cp.mindeg[i] += popc64(cadj[i]);
