@@ -151,66 +151,149 @@ __global__ void __launch_bounds__(256) vertex_core_kernel(GraphDev G, const Core
 }
 
 // ------------------------------------------------------------------------
-// 2-vertex (edge) cores: ONE LANE PER ROOT EDGE.  The Venn diagram of an edge
-// core is {|e(u)\e(v)|, |e(v)\e(u)|, |e(u)&e(v)|} = {du-1-c, dv-1-c, c} with
-// c = |N(u) & N(v)| (u, v are not in N(u) & N(v); v in N(u)).  A lane merges
-// (or gallops through) the two sorted lists itself when the shorter list has
-// <= HEAVY entries; heavier roots are ballot-collected and processed by the
-// whole warp one after another (Listing 7's "all lanes process the first such
-// vertex together"), lanes over the shorter list binary-searching the longer.
-// fc is Sec. 3.1's closed form (the paper's specialised 2-core code).
+// 2-vertex (edge) cores, two streaming passes per count:
+//
+// (A) support_kernel: c(e) = |N(u) & N(v)| for every edge e = (u < v), by
+//     listing each triangle u < v < w exactly once from its lowest edge:
+//     w in N+(u) & N+(v), N+(x) = neighbours with a larger (degree-ordered)
+//     id -- short lists, O(m^1.5) total.  The lane owning (u,v) adds its
+//     triangles to c(uv); c(uw), c(vw) receive atomics (their oriented
+//     indices come from the match positions).  One lane per root edge;
+//     roots whose shorter out-list exceeds kHeavy are collected by ballot and
+//     processed by the whole warp (Listing 7 style).
+// (B) edge_fc_kernel: lane per root edge, Venn = {du-1-c, dv-1-c, c}
+//     (e(x) excludes u and v; v in N(u); u, v not in N(u) & N(v)), fc by
+//     Sec. 3.1's closed form for every program; coalesced reads only.
 constexpr int kHeavy = 32;
 
-__device__ __forceinline__ int intersect_seq(const int32_t* __restrict__ A, int na, const int32_t* __restrict__ B,
-                                             int nb) {
-    if (na > nb) { const int32_t* t = A; A = B; B = t; int x = na; na = nb; nb = x; }
+struct OrientDev {
+    const int64_t* __restrict__ split;
+    const int64_t* __restrict__ oofs;
+};
+
+__device__ __forceinline__ int64_t oidx(const OrientDev& O, int u, int64_t p) {
+    return __ldg(O.oofs + u) + (p - __ldg(O.split + u));
+}
+
+// sequential merge / gallop of A = adj[a0, a0+na) and B = adj[b0, b0+nb);
+// every common element: atomics on the oriented edges (ua, A-pos), (ub, B-pos)
+__device__ __forceinline__ int support_seq(const int32_t* __restrict__ adj, const OrientDev& O, int ua, int64_t a0,
+                                           int na, int ub, int64_t b0, int nb, int* __restrict__ sup) {
+    if (na == 0 || nb == 0) return 0;
+    if (na > nb) {
+        int t = ua; ua = ub; ub = t;
+        int64_t t0 = a0; a0 = b0; b0 = t0;
+        int tn = na; na = nb; nb = tn;
+    }
+    const int64_t baseA = __ldg(O.oofs + ua) - __ldg(O.split + ua) ;
+    const int64_t baseB = __ldg(O.oofs + ub) - __ldg(O.split + ub);
     int c = 0;
-    if (na == 0) return 0;
-    if (nb > 8 * na) {                      // galloping search of A's elements in B
+    if (nb > 8 * na) {                       // gallop A's elements through B
         int j = 0;
         for (int i = 0; i < na && j < nb; ++i) {
-            const int x = __ldg(A + i);
+            const int x = __ldg(adj + a0 + i);
             int step = 1, hi = j;
-            while (hi < nb && __ldg(B + hi) < x) { j = hi + 1; hi += step; step <<= 1; }
+            while (hi < nb && __ldg(adj + b0 + hi) < x) { j = hi + 1; hi += step; step <<= 1; }
             if (hi > nb) hi = nb;
-            int lo = j;                      // B[lo-1] < x, search [lo, hi]
-            int h2 = hi;
+            int lo = j, h2 = hi;
             while (lo < h2) {
                 int mid = (lo + h2) >> 1;
-                if (__ldg(B + mid) < x) lo = mid + 1; else h2 = mid;
+                if (__ldg(adj + b0 + mid) < x) lo = mid + 1; else h2 = mid;
             }
             j = lo;
-            if (j < nb && __ldg(B + j) == x) { ++c; ++j; }
+            if (j < nb && __ldg(adj + b0 + j) == x) {
+                ++c;
+                atomicAdd(sup + baseA + a0 + i, 1);
+                atomicAdd(sup + baseB + b0 + j, 1);
+                ++j;
+            }
         }
         return c;
     }
-    int i = 0, j = 0;                        // linear merge
-    int a = __ldg(A), b = __ldg(B);
+    int i = 0, j = 0;
+    int x = __ldg(adj + a0), y = __ldg(adj + b0);
     for (;;) {
-        if (a < b) { if (++i == na) break; a = __ldg(A + i); }
-        else if (a > b) { if (++j == nb) break; b = __ldg(B + j); }
+        if (x < y) { if (++i == na) break; x = __ldg(adj + a0 + i); }
+        else if (x > y) { if (++j == nb) break; y = __ldg(adj + b0 + j); }
         else {
             ++c;
+            atomicAdd(sup + baseA + a0 + i, 1);
+            atomicAdd(sup + baseB + b0 + j, 1);
             if (++i == na || ++j == nb) break;
-            a = __ldg(A + i);
-            b = __ldg(B + j);
+            x = __ldg(adj + a0 + i);
+            y = __ldg(adj + b0 + j);
         }
     }
     return c;
 }
 
-// whole warp: |A & B|, lanes over the shorter list, binary search in the longer
-__device__ __forceinline__ int intersect_warp(const int32_t* __restrict__ A, int na, const int32_t* __restrict__ B,
-                                              int nb, int lane) {
-    if (na > nb) { const int32_t* t = A; A = B; B = t; int x = na; na = nb; nb = x; }
+// whole warp: lanes over the shorter list, binary search in the longer
+__device__ __forceinline__ int support_warp(const int32_t* __restrict__ adj, const OrientDev& O, int ua, int64_t a0,
+                                            int na, int ub, int64_t b0, int nb, int* __restrict__ sup, int lane) {
+    if (na > nb) {
+        int t = ua; ua = ub; ub = t;
+        int64_t t0 = a0; a0 = b0; b0 = t0;
+        int tn = na; na = nb; nb = tn;
+    }
+    const int64_t baseA = __ldg(O.oofs + ua) - __ldg(O.split + ua);
+    const int64_t baseB = __ldg(O.oofs + ub) - __ldg(O.split + ub);
     int c = 0;
-    for (int b0 = 0; b0 < na; b0 += 32) {
-        const int i = b0 + lane;
+    for (int s0 = 0; s0 < na; s0 += 32) {
+        const int i = s0 + lane;
         bool hit = false;
-        if (i < na) hit = contains(B, nb, __ldg(A + i));
+        if (i < na) {
+            const int x = __ldg(adj + a0 + i);
+            int lo = 0, hi = nb;
+            while (lo < hi) {
+                int mid = (lo + hi) >> 1;
+                if (__ldg(adj + b0 + mid) < x) lo = mid + 1; else hi = mid;
+            }
+            if (lo < nb && __ldg(adj + b0 + lo) == x) {
+                hit = true;
+                atomicAdd(sup + baseA + a0 + i, 1);
+                atomicAdd(sup + baseB + b0 + lo, 1);
+            }
+        }
         c += __popc(__ballot_sync(FULLMASK, hit));
     }
     return c;
+}
+
+__global__ void __launch_bounds__(256) support_kernel(GraphDev G, OrientDev O, int64_t m, int* __restrict__ sup,
+                                                      unsigned long long* queue) {
+    const int lane = threadIdx.x & 31;
+    for (;;) {
+        unsigned long long jq = 0;
+        if (lane == 0) jq = atomicAdd(queue, 1ull);
+        jq = __shfl_sync(FULLMASK, jq, 0);
+        const int64_t t0 = (int64_t)jq * 32;
+        if (t0 >= m) break;
+        const int64_t t = t0 + lane;
+        const bool valid = t < m;
+        const int64_t e = valid ? m - 1 - t : 0;     // heavy (high-id) roots first
+        int u = 0, v = 0, nu = 0, nv = 0;
+        int64_t su = 0, sv = 0;
+        if (valid) {
+            u = __ldg(G.osrc + e);
+            v = __ldg(G.odst + e);
+            su = __ldg(O.split + u); nu = (int)(__ldg(G.offs + u + 1) - su);
+            sv = __ldg(O.split + v); nv = (int)(__ldg(G.offs + v + 1) - sv);
+        }
+        const bool heavy = valid && min(nu, nv) > kHeavy;
+        int c = 0;
+        if (valid && !heavy) c = support_seq(G.adj, O, u, su, nu, v, sv, nv, sup);
+        unsigned hb = __ballot_sync(FULLMASK, heavy);
+        while (hb) {
+            const int who = __ffs(hb) - 1;
+            hb &= hb - 1;
+            const int wu = __shfl_sync(FULLMASK, u, who), wv = __shfl_sync(FULLMASK, v, who);
+            const int64_t wsu = __shfl_sync(FULLMASK, su, who), wsv = __shfl_sync(FULLMASK, sv, who);
+            const int wnu = __shfl_sync(FULLMASK, nu, who), wnv = __shfl_sync(FULLMASK, nv, who);
+            const int cc = support_warp(G.adj, O, wu, wsu, wnu, wv, wsv, wnv, sup, lane);
+            if (lane == who) c = cc;
+        }
+        if (valid && c) atomicAdd(sup + e, c);
+    }
 }
 
 template <class A>
@@ -225,8 +308,9 @@ __device__ __forceinline__ void edge_programs(const CoreProg& P, uint64_t nu, ui
     }
 }
 
-__global__ void __launch_bounds__(256) edge_core_kernel(GraphDev G, const CoreProg P, WorkDesc W, AccDev* acc,
-                                                        unsigned long long* matches, unsigned long long* queue) {
+__global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, const CoreProg P, WorkDesc W,
+                                                      const int* __restrict__ sup, AccDev* acc,
+                                                      unsigned long long* matches) {
     const int lane = threadIdx.x & 31;
     u128 acc_l[FSGC_MAXPATS];
     for (int i = 0; i < FSGC_MAXPATS; ++i) acc_l[i] = 0;
@@ -235,44 +319,43 @@ __global__ void __launch_bounds__(256) edge_core_kernel(GraphDev G, const CorePr
     int Kmax = 0;
     for (int pi = 0; pi < P.nprog; ++pi) Kmax = max(Kmax, (int)P.prog[pi].ksum);
     const int64_t total = W.end - W.begin;
-    for (;;) {
-        unsigned long long jq = 0;
-        if (lane == 0) jq = atomicAdd(queue, 1ull);
-        jq = __shfl_sync(FULLMASK, jq, 0);
-        const int64_t g = (int64_t)jq * W.nshards + W.shard;
-        const int64_t t0 = g * 32;
-        if (t0 >= total) break;
-        const int64_t t = t0 + lane;
-        bool active = t < total;
-        int u = 0, v = 0;
-        int64_t ou = 0, ov = 0;
-        int du = 0, dv = 0;
-        if (active) {
-            const int64_t item = W.end - 1 - t;          // heavy roots first
-            if (P.root_mode == ROOT_ORIENTED) { u = __ldg(G.osrc + item); v = __ldg(G.odst + item); }
-            else { u = __ldg(G.row + item); v = __ldg(G.adj + item); }
-            ou = __ldg(G.offs + u); du = (int)(__ldg(G.offs + u + 1) - ou);
-            ov = __ldg(G.offs + v); dv = (int)(__ldg(G.offs + v + 1) - ov);
-            if (W.degfilter && (du < P.mindeg[0] || dv < P.mindeg[1])) active = false;
+    const int64_t nchunks = (total + 31) / 32;
+    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t c0 = warp; ; c0 += nwarps) {          // chunks dealt round-robin to shards
+        const int64_t g = c0 * W.nshards + W.shard;
+        if (g >= nchunks) break;
+        const int64_t t = g * 32 + lane;
+        if (t >= total) continue;
+        const int64_t item = W.begin + t;
+        int u, v;
+        int64_t e;
+        if (P.root_mode == ROOT_ORIENTED) {
+            e = item;
+            u = __ldg(G.osrc + e);
+            v = __ldg(G.odst + e);
+        } else {                                         // directed CSR entry
+            u = __ldg(G.row + item);
+            v = __ldg(G.adj + item);
+            if (u < v) {
+                e = oidx(O, u, item);
+            } else {                                     // position of u in N+(v)
+                int64_t lo = __ldg(O.split + v), hi = __ldg(G.offs + v + 1);
+                while (lo < hi) {
+                    int64_t mid = (lo + hi) >> 1;
+                    if (__ldg(G.adj + mid) < u) lo = mid + 1; else hi = mid;
+                }
+                e = oidx(O, v, lo);
+            }
         }
-        const bool heavy = active && min(du, dv) > kHeavy;
-        int c = 0;
-        if (active && !heavy) c = intersect_seq(G.adj + ou, du, G.adj + ov, dv);
-        unsigned hb = __ballot_sync(FULLMASK, heavy);
-        while (hb) {
-            const int who = __ffs(hb) - 1;
-            hb &= hb - 1;
-            const int64_t wou = __shfl_sync(FULLMASK, ou, who), wov = __shfl_sync(FULLMASK, ov, who);
-            const int wdu = __shfl_sync(FULLMASK, du, who), wdv = __shfl_sync(FULLMASK, dv, who);
-            const int cc = intersect_warp(G.adj + wou, wdu, G.adj + wov, wdv, lane);
-            if (lane == who) c = cc;
-        }
-        if (active) {
-            ++nmatch;
-            const uint64_t nu = du - 1 - c, nv = dv - 1 - c, nuv = c;
-            if (fits64(nu + nv + nuv, Kmax)) edge_programs<Exact64>(P, nu, nv, nuv, acc_l, ovf_mask);
-            else edge_programs<Checked128>(P, nu, nv, nuv, acc_l, ovf_mask);
-        }
+        const int du = (int)(__ldg(G.offs + u + 1) - __ldg(G.offs + u));
+        const int dv = (int)(__ldg(G.offs + v + 1) - __ldg(G.offs + v));
+        if (W.degfilter && (du < P.mindeg[0] || dv < P.mindeg[1])) continue;
+        ++nmatch;
+        const uint64_t c = (uint64_t)__ldg(sup + e);
+        const uint64_t nu = du - 1 - c, nv = dv - 1 - c;
+        if (fits64(nu + nv + c, Kmax)) edge_programs<Exact64>(P, nu, nv, c, acc_l, ovf_mask);
+        else edge_programs<Checked128>(P, nu, nv, c, acc_l, ovf_mask);
     }
     warp_flush_acc(P.npats, acc_l, ovf_mask, nmatch, acc, matches, lane);
 }
@@ -600,16 +683,25 @@ extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, 
                 vertex_core_kernel<<<(int)grid, 256, 0, st>>>(G, cp, W, dacc, dmatch);
                 FSGC_CUDA(cudaGetLastError());
             } else if (cp.p == 2) {
+                // (A) per-edge common-neighbour counts, (B) fringe counts
+                DevBuf<int> sup;
+                FSGC_CUDA(sup.alloc(g->m > 0 ? g->m : 1, st));
+                FSGC_CUDA(cudaMemsetAsync(sup.ptr, 0, sizeof(int) * (g->m > 0 ? g->m : 1), st));
+                OrientDev O{g->split, g->oofs};
                 int per_sm = 0;
-                FSGC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, edge_core_kernel, 256, 0));
-                if (per_sm < 1) per_sm = 1;
-                W.chunk = 32;
-                int64_t nchunks = ((e - b) + 31) / 32;
-                int64_t mine = (nchunks + opts.shard_count - 1) / opts.shard_count;
-                int64_t grid = std::min<int64_t>((int64_t)sm_count() * per_sm, (mine + 7) / 8);
+                FSGC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, support_kernel, 256, 0));
+                int64_t grid = std::min<int64_t>((int64_t)sm_count() * std::max(per_sm, 1), (g->m + 255) / 256);
                 if (grid < 1) grid = 1;
-                edge_core_kernel<<<(int)grid, 256, 0, st>>>(G, cp, W, dacc, dmatch, dqueue);
+                support_kernel<<<(int)grid, 256, 0, st>>>(G, O, g->m, sup.ptr, dqueue);
                 FSGC_CUDA(cudaGetLastError());
+                FSGC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, edge_fc_kernel, 256, 0));
+                int64_t mine = ((e - b) + 31) / 32;
+                mine = (mine + opts.shard_count - 1) / opts.shard_count;
+                grid = std::min<int64_t>((int64_t)sm_count() * std::max(per_sm, 1), (mine + 7) / 8);
+                if (grid < 1) grid = 1;
+                edge_fc_kernel<<<(int)grid, 256, 0, st>>>(G, O, cp, W, sup.ptr, dacc, dmatch);
+                FSGC_CUDA(cudaGetLastError());
+                launches = 2;
             } else {
                 const size_t smem = (size_t)kWarps * 33 * (1u << cp.q) * sizeof(uint32_t);
                 static bool attr_set = false;

@@ -98,6 +98,23 @@ __global__ void split_keys(const uint64_t* __restrict__ keys, int64_t M, int B,
     }
 }
 
+// split[v] = first CSR position in v's list holding a neighbour > v;
+// out[v] = number of such neighbours (the degree-oriented out-degree)
+__global__ void split_points(const int64_t* __restrict__ offs, const int32_t* __restrict__ adj, int64_t n,
+                             int64_t* __restrict__ split, int64_t* __restrict__ out) {
+    for (int64_t v = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; v < n;
+         v += (int64_t)gridDim.x * blockDim.x) {
+        int64_t lo = offs[v], hi = offs[v + 1];
+        const int64_t end = hi;
+        while (lo < hi) {
+            int64_t mid = (lo + hi) >> 1;
+            if (adj[mid] <= (int32_t)v) lo = mid + 1; else hi = mid;
+        }
+        split[v] = lo;
+        out[v] = end - lo;
+    }
+}
+
 struct UpperTri {
     int B;
     uint64_t mask;
@@ -255,6 +272,19 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
         split_keys<<<grid_for(m), 256, 0, st>>>(spare, m, B, osrc.ptr, odst.ptr);
         FSGC_CUDA(cudaGetLastError());
     }
+    // oriented view: split points + exclusive scan of out-degrees
+    DevBuf<int64_t> split, oofs;
+    FSGC_CUDA(split.alloc(n, st));
+    FSGC_CUDA(oofs.alloc(n + 1, st));
+    FSGC_CUDA(cudaMemsetAsync(oofs.ptr + n, 0, sizeof(int64_t), st));
+    split_points<<<grid_for(n), 256, 0, st>>>(offs.ptr, adj.ptr, n, split.ptr, oofs.ptr);
+    FSGC_CUDA(cudaGetLastError());
+    {
+        size_t b = 0;
+        FSGC_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, b, oofs.ptr, oofs.ptr, n + 1, st));
+        if (b > tmp_bytes) { FSGC_CUDA(tmp.alloc(b, st)); tmp_bytes = b; }
+        FSGC_CUDA(cub::DeviceScan::ExclusiveSum(tmp.ptr, b, oofs.ptr, oofs.ptr, n + 1, st));
+    }
     tmp.release();
     ka.release();
     kb.release();
@@ -278,6 +308,8 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
     g->osrc = osrc.take();
     g->odst = odst.take();
     g->order = order.take();
+    g->split = split.take();
+    g->oofs = oofs.take();
     g->device = dev;
     *out = g;
     return FSGC_OK;
@@ -313,5 +345,7 @@ extern "C" void fsgc_free_graph(fsgc_graph* g) {
     cudaFree(g->osrc);
     cudaFree(g->odst);
     cudaFree(g->order);
+    cudaFree(g->split);
+    cudaFree(g->oofs);
     delete g;
 }

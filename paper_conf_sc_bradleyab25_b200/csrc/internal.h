@@ -24,6 +24,10 @@ struct fsgc_graph {
     int32_t* osrc = nullptr;     // [m]
     int32_t* odst = nullptr;     // [m]
     int32_t* order = nullptr;    // [n]
+    int64_t* split = nullptr;    // [n]   CSR position of the first neighbour > v
+    int64_t* oofs = nullptr;     // [n+1] oriented offsets: oriented index of
+                                 //       CSR position p >= split[u] is
+                                 //       oofs[u] + p - split[u]
     int device = 0;
 };
 
