@@ -274,7 +274,7 @@ def main():
     time.sleep(0.2)
     ev0 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
     ev1 = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps)]
-    kms, launches = [], 0
+    kms, ams, launches = [], [], 0
     for s in range(args.steps):
         flush.fill_(s)
         torch.cuda.synchronize()
@@ -285,30 +285,48 @@ def main():
         ev1[s].record(stream)
         torch.cuda.synchronize()
         kms.append(res[0].kernel_ms)
+        ams.append(res[0].aux_ms)
         launches += res[0].kernel_launches
     step_ms = [a.elapsed_time(b) for a, b in zip(ev0, ev1)]
     clocks = sampler.stop()
     total_ms = sum(step_ms)
     if world > 1:
-        t = torch.tensor([total_ms, sum(kms)], dtype=torch.float64, device=dev)
+        t = torch.tensor([total_ms, sum(kms), sum(ams)], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        total_ms, kms_sum = t.tolist()
+        total_ms, kms_sum, ams_sum = t.tolist()
     else:
-        kms_sum = sum(kms)
+        kms_sum, ams_sum = sum(kms), sum(ams)
     ms_per_step = total_ms / args.steps
     value = core_matches / (ms_per_step / 1e3)
     kernel_ms = kms_sum / args.steps
+    aux_ms = ams_sum / args.steps
 
-    # ---- roofline of the dominant kernel (edge-core pass: DESIGN.md)
-    offs, _, _ = g.download()
-    deg = np.diff(offs).astype(np.float64)
+    # ---- roofline of the dominant kernel: algorithmic
+    # bytes per launch / CUDA-event duration, against the measured HBM peak
+    offs, adj_h, _ = g.download()
+    deg = np.diff(offs).astype(np.int64)
+    rows = np.repeat(np.arange(n, dtype=np.int64), deg)
+    up = adj_h.astype(np.int64) > rows
+    out = np.bincount(rows[up], minlength=n).astype(np.float64)
+    indeg = deg - out
     m = g.m
-    alg_bytes = 40.0 * m + 4.0 * float((deg * deg).sum())    # per launch, all root edges
-    if world > 1:
-        alg_bytes /= world
-    achieved = alg_bytes / (kernel_ms / 1e3) / 1e9
+    share = 1.0 / world
+    # support pass: per oriented edge 8 B (u,v) + 32 B (split/offs of u and v)
+    # + 4 B per out-list entry read by the merge (out(u) + out(v)); all edges
+    sup_bytes = 40.0 * m + 4.0 * float((out * out).sum() + (indeg * out).sum())
+    # fc pass: per root edge 8 B (u,v) + 32 B (4 offsets) + 4 B support
+    fc_bytes = 44.0 * m * share
+    kernels = [("edge_fc_kernel (Venn + Sec. 3.1 fc, lane per root edge)", fc_bytes, kernel_ms),
+               ("support_kernel (per-edge |N(u)&N(v)| by oriented listing)", sup_bytes, aux_ms)]
+    kernels.sort(key=lambda k: -k[2])
     peak, peak_src = measured_peaks()
     traffic = ncu_traffic(args.workload)
+
+    def roof(name, byts, ms, traffic=None):
+        ach = byts / (ms / 1e3) / 1e9 if ms > 0 else 0.0
+        return {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
+                "traffic": traffic, "kernel": name, "kernel_ms": ms,
+                "algorithmic_bytes_per_launch": byts, "peak_source": peak_src}
 
     # ---- e2e through the public API from pinned host buffers
     e2e = None
@@ -362,10 +380,8 @@ def main():
                        "parallelism": f"{world} GPU(s): graph replicated, root-edge chunks dealt "
                                       f"round-robin, 1 all-reduce of 128-bit partials"},
             "gpu_launches": launches,
-            "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic,
-                         "kernel": "core_kernel (edge-core pass)", "kernel_ms": kernel_ms,
-                         "algorithmic_bytes_per_launch": alg_bytes, "peak_source": peak_src},
+            "roofline": roof(*kernels[0], traffic=traffic),
+            "roofline_other_kernels": [roof(*k) for k in kernels[1:]],
             "clocks": clocks,
             "e2e": e2e,
             "cpu_baseline": cpu,

@@ -169,6 +169,8 @@ typedef struct {
     int32_t root_pattern_vertex; /* pattern vertex matched at the root (c0)  */
     float kernel_ms;        /* device time of this pattern's counting kernel
                                (CUDA events around the launch on `stream`)    */
+    float aux_ms;           /* device time of the auxiliary per-edge support
+                               pass (edge cores), 0 otherwise                 */
     int32_t kernel_launches;/* kernels launched for this pattern's pass       */
 } fsgc_result;
 

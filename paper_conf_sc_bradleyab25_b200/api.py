@@ -111,6 +111,7 @@ class CountResult:
     overflow: bool
     root_pattern_vertex: int
     kernel_ms: float = 0.0
+    aux_ms: float = 0.0
     kernel_launches: int = 0
 
 
@@ -184,7 +185,7 @@ def fsgc_count(graph: Graph, patterns: Sequence[Pattern], stream=None, **kw) -> 
         out.append(CountResult(
             count=(r.count.value if (whole and not r.overflow) else None), raw=r.raw.value,
             divisor=r.divisor, core_matches=r.core_matches, overflow=bool(r.overflow),
-            root_pattern_vertex=r.root_pattern_vertex, kernel_ms=r.kernel_ms,
+            root_pattern_vertex=r.root_pattern_vertex, kernel_ms=r.kernel_ms, aux_ms=r.aux_ms,
             kernel_launches=r.kernel_launches))
     return out
 

@@ -100,25 +100,97 @@ __device__ __forceinline__ void atomic_add_u128(AccDev* a, u128 v, bool ovf) {
     if (o) atomicOr(&a->ovf, 1u);
 }
 
-// per-warp epilogue: reduce the lane accumulators, one atomic per pattern
-__device__ __forceinline__ void warp_flush_acc(int npats, u128* acc_l, uint32_t ovf_mask, unsigned long long nmatch,
-                                               AccDev* acc, unsigned long long* matches, int lane) {
+// Result sink of a pass.  Reduction is contention-free: lanes -> warp
+// (shuffles) -> block (shared memory) -> one BlockPartial per block; the last
+// block to finish (ticket) sums the partials and writes the pass result.
+struct BlockPartial {
+    unsigned long long lo[FSGC_MAXPATS], hi[FSGC_MAXPATS];
+    unsigned long long matches;
+    unsigned int ovf, pad;
+};
+
+struct Sink {
+    AccDev* acc;                    // [FSGC_MAXPATS] final result
+    unsigned long long* matches;    // final core-match count
+    BlockPartial* parts;            // [gridDim.x]
+    unsigned int* ticket;
+};
+
+__device__ __noinline__ void block_publish(int npats, const u128* acc_l, uint32_t ovf_mask, unsigned long long nmatch,
+                                           const Sink S) {
+    __shared__ unsigned long long s_lo[32][FSGC_MAXPATS], s_hi[32][FSGC_MAXPATS];
+    __shared__ unsigned int s_ovf[32];
+    __shared__ unsigned long long s_m[32];
+    __shared__ int s_last;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    uint32_t om = ovf_mask;
     for (int pi = 0; pi < npats; ++pi) {
         u128 v = acc_l[pi];
-        bool o = (ovf_mask >> pi) & 1;
+        bool o = false;
         warp_reduce_u128(v, o);
-        if (lane == 0 && (v != 0 || o)) atomic_add_u128(acc + pi, v, o);
+        if (o) om |= 1u << pi;
+        if (lane == 0) { s_lo[wid][pi] = u128_lo(v); s_hi[wid][pi] = u128_hi(v); }
     }
+    om = __reduce_or_sync(FULLMASK, om);
 #pragma unroll
     for (int o = 16; o; o >>= 1) nmatch += __shfl_down_sync(FULLMASK, nmatch, o);
-    if (lane == 0 && nmatch) atomicAdd(matches, nmatch);
+    if (lane == 0) { s_ovf[wid] = om; s_m[wid] = nmatch; }
+    __syncthreads();
+    if (wid == 0) {
+        BlockPartial* bp = S.parts + blockIdx.x;
+        for (int pi = 0; pi < npats; ++pi) {
+            u128 v = lane < nw ? u128_make(s_lo[lane][pi], s_hi[lane][pi]) : (u128)0;
+            bool o = false;
+            warp_reduce_u128(v, o);
+            if (lane == 0) { bp->lo[pi] = u128_lo(v); bp->hi[pi] = u128_hi(v); if (o) s_ovf[0] |= 1u << pi; }
+        }
+        __syncwarp();
+        uint32_t bo = __reduce_or_sync(FULLMASK, lane < nw ? s_ovf[lane] : 0u);
+        unsigned long long bm = lane < nw ? s_m[lane] : 0ull;
+#pragma unroll
+        for (int o = 16; o; o >>= 1) bm += __shfl_down_sync(FULLMASK, bm, o);
+        if (lane == 0) {
+            bp->ovf = bo;
+            bp->matches = bm;
+            __threadfence();
+            const unsigned t = atomicAdd(S.ticket, 1u);
+            s_last = (t == gridDim.x - 1);
+        }
+    }
+    __syncthreads();
+    if (s_last && wid == 0) {
+        __threadfence();
+        const int nb = gridDim.x;
+        uint32_t fo = 0;
+        unsigned long long fm = 0;
+        for (int b = lane; b < nb; b += 32) {
+            fo |= __ldcg(&S.parts[b].ovf);
+            fm += __ldcg(&S.parts[b].matches);
+        }
+        fo = __reduce_or_sync(FULLMASK, fo);
+#pragma unroll
+        for (int o = 16; o; o >>= 1) fm += __shfl_down_sync(FULLMASK, fm, o);
+        for (int pi = 0; pi < npats; ++pi) {
+            u128 v = 0;
+            bool o = false;
+            for (int b = lane; b < nb; b += 32)
+                v = add_ovf(v, u128_make(__ldcg(&S.parts[b].lo[pi]), __ldcg(&S.parts[b].hi[pi])), o);
+            warp_reduce_u128(v, o);
+            if (lane == 0) {
+                S.acc[pi].lo = u128_lo(v);
+                S.acc[pi].hi = u128_hi(v);
+                S.acc[pi].ovf = (o || ((fo >> pi) & 1)) ? 1u : 0u;
+            }
+        }
+        if (lane == 0) *S.matches = fm;
+    }
 }
 
 // ------------------------------------------------------------------------
 // 1-vertex cores (k-stars, the 1- and 2-vertex patterns): one thread per
 // root vertex, Venn = {deg(v)} (Sec. 3 k-star formula generalised by fc).
 __global__ void __launch_bounds__(256) vertex_core_kernel(GraphDev G, const CoreProg P, WorkDesc W,
-                                                          AccDev* acc, unsigned long long* matches) {
+                                                          const Sink S) {
     const int lane = threadIdx.x & 31;
     u128 acc_l[FSGC_MAXPATS];
     for (int i = 0; i < FSGC_MAXPATS; ++i) acc_l[i] = 0;
@@ -147,7 +219,7 @@ __global__ void __launch_bounds__(256) vertex_core_kernel(GraphDev G, const Core
             if (o) ovf_mask |= 1u << fp.pat;
         }
     }
-    warp_flush_acc(P.npats, acc_l, ovf_mask, nmatch, acc, matches, lane);
+    block_publish(P.npats, acc_l, ovf_mask, nmatch, S);
 }
 
 // ------------------------------------------------------------------------
@@ -309,8 +381,7 @@ __device__ __forceinline__ void edge_programs(const CoreProg& P, uint64_t nu, ui
 }
 
 __global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, const CoreProg P, WorkDesc W,
-                                                      const int* __restrict__ sup, AccDev* acc,
-                                                      unsigned long long* matches) {
+                                                      const int* __restrict__ sup, const Sink S) {
     const int lane = threadIdx.x & 31;
     u128 acc_l[FSGC_MAXPATS];
     for (int i = 0; i < FSGC_MAXPATS; ++i) acc_l[i] = 0;
@@ -357,15 +428,14 @@ __global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, c
         if (fits64(nu + nv + c, Kmax)) edge_programs<Exact64>(P, nu, nv, c, acc_l, ovf_mask);
         else edge_programs<Checked128>(P, nu, nv, c, acc_l, ovf_mask);
     }
-    warp_flush_acc(P.npats, acc_l, ovf_mask, nmatch, acc, matches, lane);
+    block_publish(P.npats, acc_l, ovf_mask, nmatch, S);
 }
 
 // ------------------------------------------------------------------------
 // Cores with p >= 2 vertices: one warp per root edge.
 template <int WARPS>
 __global__ void __launch_bounds__(WARPS * 32) core_kernel(GraphDev G, const CoreProg P, WorkDesc W,
-                                                          AccDev* acc, unsigned long long* matches,
-                                                          unsigned long long* queue) {
+                                                          const Sink S, unsigned long long* queue) {
     extern __shared__ uint32_t smem[];
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     const int q = P.q, V = 1 << q, p = P.p;
@@ -528,7 +598,7 @@ __global__ void __launch_bounds__(WARPS * 32) core_kernel(GraphDev G, const Core
         }
     }
     if (nbuf) flush();
-    warp_flush_acc(P.npats, acc_l, ovf_mask, nmatch, acc, matches, lane);
+    block_publish(P.npats, acc_l, ovf_mask, nmatch, S);
 }
 
 int sm_count() {
@@ -543,6 +613,33 @@ int sm_count() {
 }
 
 constexpr int kWarps = 4;
+
+struct LaunchCfg {
+    int vertex = 1, support = 1, edge = 1;
+    int core[FSGC_MAXQ + 1] = {};
+};
+
+const LaunchCfg& launch_cfg() {
+    static LaunchCfg L;
+    static bool init = false;
+    if (!init) {
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&L.vertex, vertex_core_kernel, 256, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&L.support, support_kernel, 256, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&L.edge, edge_fc_kernel, 256, 0);
+        cudaFuncSetAttribute(core_kernel<kWarps>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)(kWarps * 33 * (1u << FSGC_MAXQ) * sizeof(uint32_t)));
+        for (int q = 0; q <= FSGC_MAXQ; ++q) {
+            size_t smem = (size_t)kWarps * 33 * (1u << q) * sizeof(uint32_t);
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&L.core[q], core_kernel<kWarps>, kWarps * 32, smem);
+            L.core[q] = std::max(L.core[q], 1);
+        }
+        L.vertex = std::max(L.vertex, 1);
+        L.support = std::max(L.support, 1);
+        L.edge = std::max(L.edge, 1);
+        init = true;
+    }
+    return L;
+}
 
 }  // namespace
 
@@ -655,81 +752,83 @@ extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, 
         if (b > e) b = e;
 
         const int npm = (int)members.size();
-        DevBuf<unsigned char> scratch;
-        const size_t acc_bytes = sizeof(AccDev) * FSGC_MAXPATS;
-        FSGC_CUDA(scratch.alloc(acc_bytes + 64, st));
-        AccDev* dacc = (AccDev*)scratch.ptr;
-        unsigned long long* dmatch = (unsigned long long*)(scratch.ptr + acc_bytes);
-        unsigned long long* dqueue = dmatch + 1;
-        FSGC_CUDA(cudaMemsetAsync(scratch.ptr, 0, acc_bytes + 64, st));
-
         GraphDev G{g->offsets, g->adj, g->row, g->osrc, g->odst};
+        OrientDev O{g->split, g->oofs};
         WorkDesc W{b, e, opts.shard_index, opts.shard_count, 4,
                    (opts.flags & FSGC_FLAG_NO_DEGREE_FILTER) ? 0 : 1};
-        static thread_local cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+        static const LaunchCfg& L = launch_cfg();
+        const int nsm = sm_count();
+
+        // grids
+        int64_t grid = 1, grid_sup = 1;
+        size_t smem = 0;
+        const bool edge = cp.root_mode != ROOT_VERTEX && cp.p == 2;
+        if (cp.root_mode == ROOT_VERTEX) {
+            W.chunk = 256;
+            int64_t work = (e - b + opts.shard_count - 1) / opts.shard_count;
+            grid = std::max<int64_t>(1, std::min<int64_t>((work + 255) / 256, (int64_t)nsm * L.vertex));
+        } else if (edge) {
+            grid_sup = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * L.support, (g->m + 255) / 256));
+            int64_t mine = ((e - b) + 31) / 32;
+            mine = (mine + opts.shard_count - 1) / opts.shard_count;
+            grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * L.edge, (mine + 7) / 8));
+        } else {
+            smem = (size_t)kWarps * 33 * (1u << cp.q) * sizeof(uint32_t);
+            int64_t nchunks = ((e - b) + W.chunk - 1) / W.chunk;
+            int64_t mine = (nchunks + opts.shard_count - 1) / opts.shard_count;
+            grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * L.core[cp.q], (mine + kWarps - 1) / kWarps));
+        }
+
+        // one scratch allocation: header | support (edge cores) | block partials
+        const size_t hdr = 1024;
+        const size_t sup_bytes = edge ? (size_t)std::max<int64_t>(g->m, 1) * sizeof(int) : 0;
+        const size_t sup_off = hdr, parts_off = (hdr + sup_bytes + 255) & ~(size_t)255;
+        DevBuf<unsigned char> scratch;
+        FSGC_CUDA(scratch.alloc(parts_off + (size_t)grid * sizeof(BlockPartial), st));
+        FSGC_CUDA(cudaMemsetAsync(scratch.ptr, 0, hdr + sup_bytes, st));
+        AccDev* dacc = (AccDev*)scratch.ptr;                               // 16 x 32 B
+        unsigned long long* dmatch = (unsigned long long*)(scratch.ptr + 512);
+        unsigned long long* dqueue = dmatch + 1;
+        unsigned long long* dqueue2 = dmatch + 2;
+        unsigned int* dticket = (unsigned int*)(dmatch + 3);
+        int* dsup = (int*)(scratch.ptr + sup_off);
+        Sink S{dacc, dmatch, (BlockPartial*)(scratch.ptr + parts_off), dticket};
+
+        static thread_local cudaEvent_t ev0 = nullptr, ev1 = nullptr, ev2 = nullptr;
         if (!ev0) {
             FSGC_CUDA(cudaEventCreate(&ev0));
             FSGC_CUDA(cudaEventCreate(&ev1));
+            FSGC_CUDA(cudaEventCreate(&ev2));
         }
         int launches = 0;
         FSGC_CUDA(cudaEventRecord(ev0, st));
-        if (e > b) {
-            launches = 1;
-            if (cp.root_mode == ROOT_VERTEX) {
-                W.chunk = 256;
-                int64_t work = (e - b + opts.shard_count - 1) / opts.shard_count;
-                int64_t grid = (work + 255) / 256;
-                grid = std::max<int64_t>(1, std::min<int64_t>(grid, (int64_t)sm_count() * 8));
-                vertex_core_kernel<<<(int)grid, 256, 0, st>>>(G, cp, W, dacc, dmatch);
-                FSGC_CUDA(cudaGetLastError());
-            } else if (cp.p == 2) {
-                // (A) per-edge common-neighbour counts, (B) fringe counts
-                DevBuf<int> sup;
-                FSGC_CUDA(sup.alloc(g->m > 0 ? g->m : 1, st));
-                FSGC_CUDA(cudaMemsetAsync(sup.ptr, 0, sizeof(int) * (g->m > 0 ? g->m : 1), st));
-                OrientDev O{g->split, g->oofs};
-                int per_sm = 0;
-                FSGC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, support_kernel, 256, 0));
-                int64_t grid = std::min<int64_t>((int64_t)sm_count() * std::max(per_sm, 1), (g->m + 255) / 256);
-                if (grid < 1) grid = 1;
-                support_kernel<<<(int)grid, 256, 0, st>>>(G, O, g->m, sup.ptr, dqueue);
-                FSGC_CUDA(cudaGetLastError());
-                FSGC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, edge_fc_kernel, 256, 0));
-                int64_t mine = ((e - b) + 31) / 32;
-                mine = (mine + opts.shard_count - 1) / opts.shard_count;
-                grid = std::min<int64_t>((int64_t)sm_count() * std::max(per_sm, 1), (mine + 7) / 8);
-                if (grid < 1) grid = 1;
-                edge_fc_kernel<<<(int)grid, 256, 0, st>>>(G, O, cp, W, sup.ptr, dacc, dmatch);
-                FSGC_CUDA(cudaGetLastError());
-                launches = 2;
-            } else {
-                const size_t smem = (size_t)kWarps * 33 * (1u << cp.q) * sizeof(uint32_t);
-                static bool attr_set = false;
-                if (!attr_set) {
-                    FSGC_CUDA(cudaFuncSetAttribute(core_kernel<kWarps>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                                   (int)(kWarps * 33 * (1u << FSGC_MAXQ) * sizeof(uint32_t))));
-                    attr_set = true;
-                }
-                int per_sm = 0;
-                FSGC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, core_kernel<kWarps>, kWarps * 32, smem));
-                if (per_sm < 1) per_sm = 1;
-                int64_t nchunks = ((e - b) + W.chunk - 1) / W.chunk;
-                int64_t mine = (nchunks + opts.shard_count - 1) / opts.shard_count;
-                int64_t grid = std::min<int64_t>((int64_t)sm_count() * per_sm, (mine + kWarps - 1) / kWarps);
-                if (grid < 1) grid = 1;
-                core_kernel<kWarps><<<(int)grid, kWarps * 32, smem, st>>>(G, cp, W, dacc, dmatch, dqueue);
-                FSGC_CUDA(cudaGetLastError());
-            }
+        if (edge && g->m > 0) {   // (A) per-edge common-neighbour counts (all edges)
+            support_kernel<<<(int)grid_sup, 256, 0, st>>>(G, O, g->m, dsup, dqueue2);
+            FSGC_CUDA(cudaGetLastError());
+            ++launches;
         }
         FSGC_CUDA(cudaEventRecord(ev1, st));
+        if (e > b) {
+            ++launches;
+            if (cp.root_mode == ROOT_VERTEX) {
+                vertex_core_kernel<<<(int)grid, 256, 0, st>>>(G, cp, W, S);
+            } else if (edge) {    // (B) fringe counts per root edge
+                edge_fc_kernel<<<(int)grid, 256, 0, st>>>(G, O, cp, W, dsup, S);
+            } else {
+                core_kernel<kWarps><<<(int)grid, kWarps * 32, smem, st>>>(G, cp, W, S, dqueue);
+            }
+            FSGC_CUDA(cudaGetLastError());
+        }
+        FSGC_CUDA(cudaEventRecord(ev2, st));
         struct { AccDev acc[FSGC_MAXPATS]; unsigned long long match; } host;
         static_assert(sizeof(host) == sizeof(AccDev) * FSGC_MAXPATS + 8, "layout");
         FSGC_CUDA(cudaMemcpyAsync(&host, dacc, sizeof host, cudaMemcpyDeviceToHost, st));
         const AccDev* hacc = host.acc;
         const unsigned long long hmatch = host.match;
         FSGC_CUDA(cudaStreamSynchronize(st));
-        float kms = 0.f;
-        FSGC_CUDA(cudaEventElapsedTime(&kms, ev0, ev1));
+        float kms = 0.f, ams = 0.f;
+        FSGC_CUDA(cudaEventElapsedTime(&ams, ev0, ev1));
+        FSGC_CUDA(cudaEventElapsedTime(&kms, ev1, ev2));
         for (int mi = 0; mi < npm; ++mi) {
             fsgc_result& r = results[members[mi]];
             r.raw.lo = hacc[mi].lo;
@@ -739,6 +838,7 @@ extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, 
             r.core_matches = hmatch;
             r.root_pattern_vertex = plan.root_pattern_vertex[mi];
             r.kernel_ms = kms;
+            r.aux_ms = ams;
             r.kernel_launches = launches;
             if (opts.shard_count == 1 && opts.root_begin <= 0 && opts.root_end < 0) {
                 rc = fsgc_finalize(r.raw, r.divisor, r.overflow, &r.count, &r.overflow);

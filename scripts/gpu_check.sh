@@ -15,6 +15,6 @@ timeout 600 python bench.py --workload $WL > $OUT/bench_${TAG}_$WL.json 2> $OUT/
 cat $OUT/bench_${TAG}_$WL.json | head -c 3000; echo
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
   --log-file $OUT/launches_${TAG}_$WL.csv python bench.py --workload $WL --steps 5 --warmup 3 --no-e2e --no-cpu-baseline > /dev/null 2>&1; echo "ncu launches rc=$?"
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:core_kernel -s 3 -c 1 \
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:'support_kernel|edge_fc_kernel|core_kernel' -s 8 -c 2 \
   -o $OUT/prof_${TAG}_$WL -f python bench.py --workload $WL --steps 2 --warmup 3 --no-e2e --no-cpu-baseline > $OUT/ncu_full_${TAG}.log 2>&1; echo "ncu full rc=$?"
 ls -la $OUT
