@@ -24,6 +24,7 @@
 #include <cstring>
 #include <map>
 #include <mutex>
+#include <tuple>
 #include "devbuf.cuh"
 #include "u128.cuh"
 #include "fc.cuh"
@@ -100,6 +101,28 @@ __device__ __forceinline__ void atomic_add_u128(AccDev* a, u128 v, bool ovf) {
     if (o) atomicOr(&a->ovf, 1u);
 }
 
+// Per-lane accumulators for NP patterns, register resident (pattern index
+// resolved by an unrolled compare, never by dynamic indexing).
+template <int NP>
+struct AccN {
+    u128 v[NP];
+    uint32_t ovf;
+    __device__ __forceinline__ void init() {
+#pragma unroll
+        for (int k = 0; k < NP; ++k) v[k] = 0;
+        ovf = 0;
+    }
+    __device__ __forceinline__ void add(int pat, u128 c, bool o) {
+#pragma unroll
+        for (int k = 0; k < NP; ++k)
+            if (k == pat) {
+                bool oo = o;
+                v[k] = add_ovf(v[k], c, oo);
+                if (oo) ovf |= 1u << k;
+            }
+    }
+};
+
 // Result sink of a pass.  Reduction is contention-free: lanes -> warp
 // (shuffles) -> block (shared memory) -> one BlockPartial per block; the last
 // block to finish (ticket) sums the partials and writes the pass result.
@@ -116,16 +139,17 @@ struct Sink {
     unsigned int* ticket;
 };
 
-__device__ __noinline__ void block_publish(int npats, const u128* acc_l, uint32_t ovf_mask, unsigned long long nmatch,
-                                           const Sink S) {
-    __shared__ unsigned long long s_lo[32][FSGC_MAXPATS], s_hi[32][FSGC_MAXPATS];
+template <int NP>
+__device__ __forceinline__ void block_publish(const AccN<NP>& A, unsigned long long nmatch, const Sink S) {
+    __shared__ unsigned long long s_lo[32][NP], s_hi[32][NP];
     __shared__ unsigned int s_ovf[32];
     __shared__ unsigned long long s_m[32];
     __shared__ int s_last;
     const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = blockDim.x >> 5;
-    uint32_t om = ovf_mask;
-    for (int pi = 0; pi < npats; ++pi) {
-        u128 v = acc_l[pi];
+    uint32_t om = A.ovf;
+#pragma unroll
+    for (int pi = 0; pi < NP; ++pi) {
+        u128 v = A.v[pi];
         bool o = false;
         warp_reduce_u128(v, o);
         if (o) om |= 1u << pi;
@@ -138,14 +162,16 @@ __device__ __noinline__ void block_publish(int npats, const u128* acc_l, uint32_
     __syncthreads();
     if (wid == 0) {
         BlockPartial* bp = S.parts + blockIdx.x;
-        for (int pi = 0; pi < npats; ++pi) {
+        uint32_t bo = lane < nw ? s_ovf[lane] : 0u;
+#pragma unroll
+        for (int pi = 0; pi < NP; ++pi) {
             u128 v = lane < nw ? u128_make(s_lo[lane][pi], s_hi[lane][pi]) : (u128)0;
             bool o = false;
             warp_reduce_u128(v, o);
-            if (lane == 0) { bp->lo[pi] = u128_lo(v); bp->hi[pi] = u128_hi(v); if (o) s_ovf[0] |= 1u << pi; }
+            if (o) bo |= 1u << pi;
+            if (lane == 0) { bp->lo[pi] = u128_lo(v); bp->hi[pi] = u128_hi(v); }
         }
-        __syncwarp();
-        uint32_t bo = __reduce_or_sync(FULLMASK, lane < nw ? s_ovf[lane] : 0u);
+        bo = __reduce_or_sync(FULLMASK, bo);
         unsigned long long bm = lane < nw ? s_m[lane] : 0ull;
 #pragma unroll
         for (int o = 16; o; o >>= 1) bm += __shfl_down_sync(FULLMASK, bm, o);
@@ -158,43 +184,52 @@ __device__ __noinline__ void block_publish(int npats, const u128* acc_l, uint32_
         }
     }
     __syncthreads();
-    if (s_last && wid == 0) {
+    // last block: warp w sums pattern w (and warp 0 the flags / matches)
+    if (s_last) {
         __threadfence();
         const int nb = gridDim.x;
-        uint32_t fo = 0;
-        unsigned long long fm = 0;
-        for (int b = lane; b < nb; b += 32) {
-            fo |= __ldcg(&S.parts[b].ovf);
-            fm += __ldcg(&S.parts[b].matches);
-        }
-        fo = __reduce_or_sync(FULLMASK, fo);
+        if (wid == 0) {
+            uint32_t fo = 0;
+            unsigned long long fm = 0;
+#pragma unroll 4
+            for (int b = lane; b < nb; b += 32) {
+                fo |= __ldcg(&S.parts[b].ovf);
+                fm += __ldcg(&S.parts[b].matches);
+            }
+            fo = __reduce_or_sync(FULLMASK, fo);
 #pragma unroll
-        for (int o = 16; o; o >>= 1) fm += __shfl_down_sync(FULLMASK, fm, o);
-        for (int pi = 0; pi < npats; ++pi) {
+            for (int o = 16; o; o >>= 1) fm += __shfl_down_sync(FULLMASK, fm, o);
+            if (lane == 0) {
+                *S.matches = fm;
+                for (int pi = 0; pi < NP; ++pi) S.acc[pi].pad = fo;  // flags, folded below
+            }
+        }
+        __syncthreads();
+        for (int pi = wid; pi < NP; pi += nw) {
             u128 v = 0;
             bool o = false;
+#pragma unroll 4
             for (int b = lane; b < nb; b += 32)
                 v = add_ovf(v, u128_make(__ldcg(&S.parts[b].lo[pi]), __ldcg(&S.parts[b].hi[pi])), o);
             warp_reduce_u128(v, o);
             if (lane == 0) {
+                const uint32_t fo = S.acc[pi].pad;
                 S.acc[pi].lo = u128_lo(v);
                 S.acc[pi].hi = u128_hi(v);
                 S.acc[pi].ovf = (o || ((fo >> pi) & 1)) ? 1u : 0u;
             }
         }
-        if (lane == 0) *S.matches = fm;
     }
 }
 
 // ------------------------------------------------------------------------
 // 1-vertex cores (k-stars, the 1- and 2-vertex patterns): one thread per
 // root vertex, Venn = {deg(v)} (Sec. 3 k-star formula generalised by fc).
+template <int NP>
 __global__ void __launch_bounds__(256) vertex_core_kernel(GraphDev G, const CoreProg P, WorkDesc W,
                                                           const Sink S) {
-    const int lane = threadIdx.x & 31;
-    u128 acc_l[FSGC_MAXPATS];
-    for (int i = 0; i < FSGC_MAXPATS; ++i) acc_l[i] = 0;
-    uint32_t ovf_mask = 0;   // per-pattern overflow bits
+    AccN<NP> acc;
+    acc.init();
     unsigned long long nmatch = 0;
     const int64_t total = W.end - W.begin;
     const int64_t nchunks = (total + W.chunk - 1) / W.chunk;
@@ -215,11 +250,10 @@ __global__ void __launch_bounds__(256) vertex_core_kernel(GraphDev G, const Core
             const FringeProg fp = P.prog[pi];
             bool o = false;
             u128 c2 = fc_dispatch<4>(venn, P.q, fp, o);
-            acc_l[fp.pat] = add_ovf(acc_l[fp.pat], c2, o);
-            if (o) ovf_mask |= 1u << fp.pat;
+            acc.add(fp.pat, c2, o);
         }
     }
-    block_publish(P.npats, acc_l, ovf_mask, nmatch, S);
+    block_publish<NP>(acc, nmatch, S);
 }
 
 // ------------------------------------------------------------------------
@@ -368,24 +402,30 @@ __global__ void __launch_bounds__(256) support_kernel(GraphDev G, OrientDev O, i
     }
 }
 
-template <class A>
+// rare path (values too large for the 64-bit bound): kept out of line so the
+// common path stays register-lean
+__device__ __noinline__ u128 edge_formula_checked(uint64_t nu, uint64_t nv, uint64_t nuv, int k, int l, int m,
+                                                  bool& o) {
+    return edge_formula<Checked128>(nu, nv, nuv, k, l, m, o);
+}
+
+template <class A, int NP>
 __device__ __forceinline__ void edge_programs(const CoreProg& P, uint64_t nu, uint64_t nv, uint64_t nuv,
-                                              u128* acc_l, uint32_t& ovf_mask) {
+                                              AccN<NP>& acc) {
     for (int pi = 0; pi < P.nprog; ++pi) {
         bool o = false;
-        const int pat = P.prog[pi].pat;
-        u128 c = A::widen(edge_formula<A>(nu, nv, nuv, P.ek[pi], P.el[pi], P.em[pi], o));
-        acc_l[pat] = add_ovf(acc_l[pat], c, o);
-        if (o) ovf_mask |= 1u << pat;
+        u128 c = A::is_wide ? edge_formula_checked(nu, nv, nuv, P.ek[pi], P.el[pi], P.em[pi], o)
+                            : A::widen(edge_formula<A>(nu, nv, nuv, P.ek[pi], P.el[pi], P.em[pi], o));
+        acc.add(P.prog[pi].pat, c, o);
     }
 }
 
+template <int NP>
 __global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, const CoreProg P, WorkDesc W,
                                                       const int* __restrict__ sup, const Sink S) {
     const int lane = threadIdx.x & 31;
-    u128 acc_l[FSGC_MAXPATS];
-    for (int i = 0; i < FSGC_MAXPATS; ++i) acc_l[i] = 0;
-    uint32_t ovf_mask = 0;
+    AccN<NP> acc;
+    acc.init();
     unsigned long long nmatch = 0;
     int Kmax = 0;
     for (int pi = 0; pi < P.nprog; ++pi) Kmax = max(Kmax, (int)P.prog[pi].ksum);
@@ -425,15 +465,16 @@ __global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, c
         ++nmatch;
         const uint64_t c = (uint64_t)__ldg(sup + e);
         const uint64_t nu = du - 1 - c, nv = dv - 1 - c;
-        if (fits64(nu + nv + c, Kmax)) edge_programs<Exact64>(P, nu, nv, c, acc_l, ovf_mask);
-        else edge_programs<Checked128>(P, nu, nv, c, acc_l, ovf_mask);
+        if (fits64(nu + nv + c, Kmax)) edge_programs<Exact64, NP>(P, nu, nv, c, acc);
+        else edge_programs<Checked128, NP>(P, nu, nv, c, acc);
     }
-    block_publish(P.npats, acc_l, ovf_mask, nmatch, S);
+    (void)lane;
+    block_publish<NP>(acc, nmatch, S);
 }
 
 // ------------------------------------------------------------------------
 // Cores with p >= 2 vertices: one warp per root edge.
-template <int WARPS>
+template <int WARPS, int NP>
 __global__ void __launch_bounds__(WARPS * 32) core_kernel(GraphDev G, const CoreProg P, WorkDesc W,
                                                           const Sink S, unsigned long long* queue) {
     extern __shared__ uint32_t smem[];
@@ -442,9 +483,8 @@ __global__ void __launch_bounds__(WARPS * 32) core_kernel(GraphDev G, const Core
     uint32_t* hist = smem + wib * (V * 33);
     uint32_t* vbuf = hist + V;
     int nbuf = 0;
-    u128 acc_l[FSGC_MAXPATS];
-    for (int i = 0; i < FSGC_MAXPATS; ++i) acc_l[i] = 0;
-    uint32_t ovf_mask = 0;   // per-pattern overflow bits
+    AccN<NP> acc;
+    acc.init();
     unsigned long long nmatch = 0;
 
     int emb[FSGC_MAXC];
@@ -465,8 +505,7 @@ __global__ void __launch_bounds__(WARPS * 32) core_kernel(GraphDev G, const Core
             const FringeProg fp = P.prog[pi];
             bool o = false;
             u128 c = fc_dispatch<FSGC_FC_STACK>(vloc, q, fp, o);
-            acc_l[fp.pat] = add_ovf(acc_l[fp.pat], c, o);
-            if (o) ovf_mask |= 1u << fp.pat;
+            acc.add(fp.pat, c, o);
         }
         nbuf = 0;
         __syncwarp();
@@ -598,7 +637,7 @@ __global__ void __launch_bounds__(WARPS * 32) core_kernel(GraphDev G, const Core
         }
     }
     if (nbuf) flush();
-    block_publish(P.npats, acc_l, ovf_mask, nmatch, S);
+    block_publish<NP>(acc, nmatch, S);
 }
 
 int sm_count() {
@@ -614,31 +653,37 @@ int sm_count() {
 
 constexpr int kWarps = 4;
 
-struct LaunchCfg {
-    int vertex = 1, support = 1, edge = 1;
-    int core[FSGC_MAXQ + 1] = {};
+// resident blocks per SM of a kernel (cached per function / block / smem)
+int occupancy(const void* fn, int threads, size_t smem) {
+    static std::mutex mu;
+    static std::map<std::tuple<const void*, int, size_t>, int> cache;
+    std::lock_guard<std::mutex> lock(mu);
+    auto key = std::make_tuple(fn, threads, smem);
+    auto it = cache.find(key);
+    if (it != cache.end()) return it->second;
+    int n = 0;
+    if (smem > 48 * 1024) cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, threads, smem);
+    n = std::max(n, 1);
+    cache[key] = n;
+    return n;
+}
+
+template <int NP>
+struct Kernels {
+    static const void* vertex() { return (const void*)vertex_core_kernel<NP>; }
+    static const void* edge() { return (const void*)edge_fc_kernel<NP>; }
+    static const void* core() { return (const void*)core_kernel<kWarps, NP>; }
 };
 
-const LaunchCfg& launch_cfg() {
-    static LaunchCfg L;
-    static bool init = false;
-    if (!init) {
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&L.vertex, vertex_core_kernel, 256, 0);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&L.support, support_kernel, 256, 0);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&L.edge, edge_fc_kernel, 256, 0);
-        cudaFuncSetAttribute(core_kernel<kWarps>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)(kWarps * 33 * (1u << FSGC_MAXQ) * sizeof(uint32_t)));
-        for (int q = 0; q <= FSGC_MAXQ; ++q) {
-            size_t smem = (size_t)kWarps * 33 * (1u << q) * sizeof(uint32_t);
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&L.core[q], core_kernel<kWarps>, kWarps * 32, smem);
-            L.core[q] = std::max(L.core[q], 1);
-        }
-        L.vertex = std::max(L.vertex, 1);
-        L.support = std::max(L.support, 1);
-        L.edge = std::max(L.edge, 1);
-        init = true;
-    }
-    return L;
+// smallest NP in {1,2,4,8,16} holding npats
+int np_class(int npats) { return npats <= 1 ? 1 : npats <= 2 ? 2 : npats <= 4 ? 4 : npats <= 8 ? 8 : 16; }
+
+const void* kernel_for(int kind, int np) {
+#define FSGC_K(NPV) case NPV: return kind == 0 ? Kernels<NPV>::vertex() : kind == 1 ? Kernels<NPV>::edge() : Kernels<NPV>::core();
+    switch (np) { FSGC_K(1) FSGC_K(2) FSGC_K(4) FSGC_K(8) FSGC_K(16) }
+#undef FSGC_K
+    return nullptr;
 }
 
 }  // namespace
@@ -756,8 +801,8 @@ extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, 
         OrientDev O{g->split, g->oofs};
         WorkDesc W{b, e, opts.shard_index, opts.shard_count, 4,
                    (opts.flags & FSGC_FLAG_NO_DEGREE_FILTER) ? 0 : 1};
-        static const LaunchCfg& L = launch_cfg();
         const int nsm = sm_count();
+        const int npc = np_class(npm);
 
         // grids
         int64_t grid = 1, grid_sup = 1;
@@ -766,17 +811,21 @@ extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, 
         if (cp.root_mode == ROOT_VERTEX) {
             W.chunk = 256;
             int64_t work = (e - b + opts.shard_count - 1) / opts.shard_count;
-            grid = std::max<int64_t>(1, std::min<int64_t>((work + 255) / 256, (int64_t)nsm * L.vertex));
+            grid = std::max<int64_t>(1, std::min<int64_t>((work + 255) / 256,
+                                                          (int64_t)nsm * occupancy(kernel_for(0, npc), 256, 0)));
         } else if (edge) {
-            grid_sup = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * L.support, (g->m + 255) / 256));
+            grid_sup = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy((const void*)support_kernel, 256, 0),
+                                                              (g->m + 255) / 256));
             int64_t mine = ((e - b) + 31) / 32;
             mine = (mine + opts.shard_count - 1) / opts.shard_count;
-            grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * L.edge, (mine + 7) / 8));
+            grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy(kernel_for(1, npc), 256, 0),
+                                                          (mine + 7) / 8));
         } else {
             smem = (size_t)kWarps * 33 * (1u << cp.q) * sizeof(uint32_t);
             int64_t nchunks = ((e - b) + W.chunk - 1) / W.chunk;
             int64_t mine = (nchunks + opts.shard_count - 1) / opts.shard_count;
-            grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * L.core[cp.q], (mine + kWarps - 1) / kWarps));
+            grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy(kernel_for(2, npc), kWarps * 32, smem),
+                                                          (mine + kWarps - 1) / kWarps));
         }
 
         // one scratch allocation: header | support (edge cores) | block partials
@@ -810,12 +859,17 @@ extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, 
         FSGC_CUDA(cudaEventRecord(ev1, st));
         if (e > b) {
             ++launches;
-            if (cp.root_mode == ROOT_VERTEX) {
-                vertex_core_kernel<<<(int)grid, 256, 0, st>>>(G, cp, W, S);
-            } else if (edge) {    // (B) fringe counts per root edge
-                edge_fc_kernel<<<(int)grid, 256, 0, st>>>(G, O, cp, W, dsup, S);
+            const int kind = cp.root_mode == ROOT_VERTEX ? 0 : edge ? 1 : 2;
+            const void* fn = kernel_for(kind, npc);
+            void* args_v[] = {(void*)&G, (void*)&cp, (void*)&W, (void*)&S};
+            void* args_e[] = {(void*)&G, (void*)&O, (void*)&cp, (void*)&W, (void*)&dsup, (void*)&S};
+            void* args_c[] = {(void*)&G, (void*)&cp, (void*)&W, (void*)&S, (void*)&dqueue};
+            if (kind == 0) {
+                FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(256), args_v, 0, st));
+            } else if (kind == 1) {   // (B) fringe counts per root edge
+                FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(256), args_e, 0, st));
             } else {
-                core_kernel<kWarps><<<(int)grid, kWarps * 32, smem, st>>>(G, cp, W, S, dqueue);
+                FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(kWarps * 32), args_c, smem, st));
             }
             FSGC_CUDA(cudaGetLastError());
         }

@@ -18,6 +18,7 @@
 
 struct Exact64 {
     typedef uint64_t T;
+    static constexpr bool is_wide = false;
     static __device__ __forceinline__ T add(T a, T b, bool&) { return a + b; }
     static __device__ __forceinline__ T mul(T a, T b, bool&) { return a * b; }
     static __device__ __forceinline__ T binom(uint64_t n, uint32_t k, bool&) {
@@ -26,14 +27,26 @@ struct Exact64 {
         if (k == 1) return n;
         if (k == 2) return (n & 1) ? n * ((n - 1) >> 1) : (n >> 1) * (n - 1);
         uint64_t r = 1;
-        for (uint32_t i = 1; i <= k; ++i) r = r * (n - k + i) / i;
+        for (uint32_t i = 1; i <= k; ++i) r = exact_div(r * (n - k + i), i);
         return r;
+    }
+    // x / d for d | x (exact): shift out the 2-adic part, multiply by the
+    // inverse of the odd part mod 2^64 (Newton: 5 steps from 3 correct bits)
+    static __device__ __forceinline__ uint64_t exact_div(uint64_t x, uint32_t d) {
+        const int tz = __ffs(d) - 1;
+        x >>= tz;
+        const uint64_t od = (uint64_t)(d >> tz);
+        uint64_t inv = od;
+#pragma unroll
+        for (int it = 0; it < 5; ++it) inv *= 2 - od * inv;
+        return x * inv;
     }
     static __device__ __forceinline__ u128 widen(T x) { return (u128)x; }
 };
 
 struct Checked128 {
     typedef u128 T;
+    static constexpr bool is_wide = true;
     static __device__ __forceinline__ T add(T a, T b, bool& o) { return add_ovf(a, b, o); }
     static __device__ __forceinline__ T mul(T a, T b, bool& o) { return mul_ovf(a, b, o); }
     static __device__ __forceinline__ T binom(uint64_t n, uint32_t k, bool& o) { return binom_ovf(n, k, o); }
