@@ -409,66 +409,91 @@ __device__ __noinline__ u128 edge_formula_checked(uint64_t nu, uint64_t nv, uint
     return edge_formula<Checked128>(nu, nv, nuv, k, l, m, o);
 }
 
-template <class A, int NP>
-__device__ __forceinline__ void edge_programs(const CoreProg& P, uint64_t nu, uint64_t nv, uint64_t nuv,
-                                              AccN<NP>& acc) {
-    for (int pi = 0; pi < P.nprog; ++pi) {
-        bool o = false;
-        u128 c = A::is_wide ? edge_formula_checked(nu, nv, nuv, P.ek[pi], P.el[pi], P.em[pi], o)
-                            : A::widen(edge_formula<A>(nu, nv, nuv, P.ek[pi], P.el[pi], P.em[pi], o));
-        acc.add(P.prog[pi].pat, c, o);
+// oriented index of the directed CSR entry `item` = (u, v)
+__device__ __forceinline__ int64_t edge_of_entry(const GraphDev& G, const OrientDev& O, int u, int v, int64_t item) {
+    if (u < v) return oidx(O, u, item);
+    int64_t lo = __ldg(O.split + v), hi = __ldg(G.offs + v + 1);   // position of u in N+(v)
+    while (lo < hi) {
+        int64_t mid = (lo + hi) >> 1;
+        if (__ldg(G.adj + mid) < u) lo = mid + 1; else hi = mid;
     }
+    return oidx(O, v, lo);
 }
+
+constexpr int kEdgeILP = 4;   // root edges per lane per iteration (independent loads in flight)
 
 template <int NP>
 __global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, const CoreProg P, WorkDesc W,
                                                       const int* __restrict__ sup, const Sink S) {
+    // program table in shared memory: k | l << 8 | m << 16 | pattern << 24
+    __shared__ uint32_t s_prog[FSGC_MAXPROG];
+    __shared__ int s_kmax, s_minm;
+    if (threadIdx.x == 0) {
+        int kmax = 0, minm = 255;
+        for (int pi = 0; pi < P.nprog; ++pi) {
+            kmax = max(kmax, (int)P.prog[pi].ksum);
+            minm = min(minm, (int)P.em[pi]);
+        }
+        s_kmax = kmax;
+        s_minm = minm;
+    }
+    if (threadIdx.x < P.nprog)
+        s_prog[threadIdx.x] = P.ek[threadIdx.x] | (P.el[threadIdx.x] << 8) | (P.em[threadIdx.x] << 16) |
+                              ((uint32_t)P.prog[threadIdx.x].pat << 24);
+    __syncthreads();
+    const int nprog = P.nprog, Kmax = s_kmax;
+    const uint64_t minm = (uint64_t)s_minm;
     const int lane = threadIdx.x & 31;
     AccN<NP> acc;
     acc.init();
     unsigned long long nmatch = 0;
-    int Kmax = 0;
-    for (int pi = 0; pi < P.nprog; ++pi) Kmax = max(Kmax, (int)P.prog[pi].ksum);
     const int64_t total = W.end - W.begin;
-    const int64_t nchunks = (total + 31) / 32;
+    constexpr int SPAN = 32 * kEdgeILP;
+    const int64_t nchunks = (total + SPAN - 1) / SPAN;
     const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    const bool oriented = P.root_mode == ROOT_ORIENTED;
     for (int64_t c0 = warp; ; c0 += nwarps) {          // chunks dealt round-robin to shards
         const int64_t g = c0 * W.nshards + W.shard;
         if (g >= nchunks) break;
-        const int64_t t = g * 32 + lane;
-        if (t >= total) continue;
-        const int64_t item = W.begin + t;
-        int u, v;
-        int64_t e;
-        if (P.root_mode == ROOT_ORIENTED) {
-            e = item;
-            u = __ldg(G.osrc + e);
-            v = __ldg(G.odst + e);
-        } else {                                         // directed CSR entry
-            u = __ldg(G.row + item);
-            v = __ldg(G.adj + item);
-            if (u < v) {
-                e = oidx(O, u, item);
-            } else {                                     // position of u in N+(v)
-                int64_t lo = __ldg(O.split + v), hi = __ldg(G.offs + v + 1);
-                while (lo < hi) {
-                    int64_t mid = (lo + hi) >> 1;
-                    if (__ldg(G.adj + mid) < u) lo = mid + 1; else hi = mid;
-                }
-                e = oidx(O, v, lo);
+        int u[kEdgeILP], v[kEdgeILP];
+        int64_t e[kEdgeILP];
+        bool ok[kEdgeILP];
+#pragma unroll
+        for (int j = 0; j < kEdgeILP; ++j) {           // 1: root edges (coalesced)
+            const int64_t t = g * SPAN + j * 32 + lane;
+            ok[j] = t < total;
+            const int64_t item = W.begin + (ok[j] ? t : 0);
+            if (oriented) { u[j] = __ldg(G.osrc + item); v[j] = __ldg(G.odst + item); e[j] = item; }
+            else { u[j] = __ldg(G.row + item); v[j] = __ldg(G.adj + item); }
+        }
+        int du[kEdgeILP], dv[kEdgeILP], c[kEdgeILP];
+#pragma unroll
+        for (int j = 0; j < kEdgeILP; ++j) {           // 2: degrees + support
+            if (!oriented) e[j] = edge_of_entry(G, O, u[j], v[j], W.begin + (ok[j] ? g * SPAN + j * 32 + lane : 0));
+            du[j] = (int)(__ldg(G.offs + u[j] + 1) - __ldg(G.offs + u[j]));
+            dv[j] = (int)(__ldg(G.offs + v[j] + 1) - __ldg(G.offs + v[j]));
+            c[j] = __ldg(sup + e[j]);
+        }
+#pragma unroll
+        for (int j = 0; j < kEdgeILP; ++j) {           // 3: Venn + fc
+            if (!ok[j]) continue;
+            if (W.degfilter && (du[j] < P.mindeg[0] || dv[j] < P.mindeg[1])) continue;
+            ++nmatch;
+            const uint64_t cc = (uint64_t)c[j];
+            if (cc < minm) continue;                    // every program needs >= minm wedge fringes
+            const uint64_t nu = du[j] - 1 - cc, nv = dv[j] - 1 - cc;
+            const bool small = fits64(nu + nv + cc, Kmax);
+            for (int pi = 0; pi < nprog; ++pi) {
+                const uint32_t w = s_prog[pi];
+                const int k = w & 255, l = (w >> 8) & 255, m = (w >> 16) & 255;
+                bool o = false;
+                const u128 f = small ? (u128)edge_formula<Exact64>(nu, nv, cc, k, l, m, o)
+                                     : edge_formula_checked(nu, nv, cc, k, l, m, o);
+                acc.add((int)(w >> 24), f, o);
             }
         }
-        const int du = (int)(__ldg(G.offs + u + 1) - __ldg(G.offs + u));
-        const int dv = (int)(__ldg(G.offs + v + 1) - __ldg(G.offs + v));
-        if (W.degfilter && (du < P.mindeg[0] || dv < P.mindeg[1])) continue;
-        ++nmatch;
-        const uint64_t c = (uint64_t)__ldg(sup + e);
-        const uint64_t nu = du - 1 - c, nv = dv - 1 - c;
-        if (fits64(nu + nv + c, Kmax)) edge_programs<Exact64, NP>(P, nu, nv, c, acc);
-        else edge_programs<Checked128, NP>(P, nu, nv, c, acc);
     }
-    (void)lane;
     block_publish<NP>(acc, nmatch, S);
 }
 
