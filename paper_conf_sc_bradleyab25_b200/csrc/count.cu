@@ -140,7 +140,7 @@ struct Sink {
 };
 
 template <int NP>
-__device__ __forceinline__ void block_publish(const AccN<NP>& A, unsigned long long nmatch, const Sink S) {
+__device__ __noinline__ void block_publish(const AccN<NP> A, unsigned long long nmatch, const Sink S) {
     __shared__ unsigned long long s_lo[32][NP], s_hi[32][NP];
     __shared__ unsigned int s_ovf[32];
     __shared__ unsigned long long s_m[32];
@@ -402,10 +402,13 @@ __global__ void __launch_bounds__(256) support_kernel(GraphDev G, OrientDev O, i
     }
 }
 
-// rare path (values too large for the 64-bit bound): kept out of line so the
-// common path stays register-lean
-__device__ __noinline__ u128 edge_formula_checked(uint64_t nu, uint64_t nv, uint64_t nuv, int k, int l, int m,
-                                                  bool& o) {
+// One program of the Sec. 3.1 closed form, out of line: the kernels are short
+// and latency-bound, so a compact hot path (instruction-cache footprint)
+// matters more than call overhead.  `small`: the 64-bit bound holds.
+__device__ __noinline__ u128 edge_prog_eval(uint64_t nu, uint64_t nv, uint64_t nuv, uint32_t w, bool small,
+                                            bool& o) {
+    const int k = w & 255, l = (w >> 8) & 255, m = (w >> 16) & 255;
+    if (small) return (u128)edge_formula<Exact64>(nu, nv, nuv, k, l, m, o);
     return edge_formula<Checked128>(nu, nv, nuv, k, l, m, o);
 }
 
@@ -484,12 +487,11 @@ __global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, c
             if (cc < minm) continue;                    // every program needs >= minm wedge fringes
             const uint64_t nu = du[j] - 1 - cc, nv = dv[j] - 1 - cc;
             const bool small = fits64(nu + nv + cc, Kmax);
+#pragma unroll 1
             for (int pi = 0; pi < nprog; ++pi) {
                 const uint32_t w = s_prog[pi];
-                const int k = w & 255, l = (w >> 8) & 255, m = (w >> 16) & 255;
                 bool o = false;
-                const u128 f = small ? (u128)edge_formula<Exact64>(nu, nv, cc, k, l, m, o)
-                                     : edge_formula_checked(nu, nv, cc, k, l, m, o);
+                const u128 f = edge_prog_eval(nu, nv, cc, w, small, o);
                 acc.add((int)(w >> 24), f, o);
             }
         }
