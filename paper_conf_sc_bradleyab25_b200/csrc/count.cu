@@ -25,6 +25,8 @@
 #include <map>
 #include <mutex>
 #include <tuple>
+#include <string>
+#include <cstdlib>
 #include "devbuf.cuh"
 #include "u128.cuh"
 #include "fc.cuh"
@@ -137,6 +139,7 @@ struct Sink {
     unsigned long long* matches;    // final core-match count
     BlockPartial* parts;            // [gridDim.x]
     unsigned int* ticket;
+    int mode;                       // 0: partials + last block sums; 1: one atomic per block
 };
 
 template <int NP>
@@ -175,6 +178,14 @@ __device__ __noinline__ void block_publish(const AccN<NP> A, unsigned long long 
         unsigned long long bm = lane < nw ? s_m[lane] : 0ull;
 #pragma unroll
         for (int o = 16; o; o >>= 1) bm += __shfl_down_sync(FULLMASK, bm, o);
+        if (S.mode == 1) {               // block totals straight into the result
+            if (lane < NP) {
+                const u128 v = u128_make(bp->lo[lane], bp->hi[lane]);
+                if (v != 0 || ((bo >> lane) & 1)) atomic_add_u128(S.acc + lane, v, (bo >> lane) & 1);
+            }
+            if (lane == 0 && bm) atomicAdd(S.matches, bm);
+            return;                      // uniform per block: s_last never set
+        }
         if (lane == 0) {
             bp->ovf = bo;
             bp->matches = bm;
@@ -183,6 +194,7 @@ __device__ __noinline__ void block_publish(const AccN<NP> A, unsigned long long 
             s_last = (t == gridDim.x - 1);
         }
     }
+    if (S.mode == 1) return;
     __syncthreads();
     // last block: warp w sums pattern w (and warp 0 the flags / matches)
     if (s_last) {
@@ -680,6 +692,20 @@ int sm_count() {
 
 constexpr int kWarps = 4;
 
+// tuning knobs (environment, read once): experiments only, defaults are the
+// tuned values
+int tune(const char* name, int dflt) {
+    static std::mutex mu;
+    static std::map<std::string, int> cache;
+    std::lock_guard<std::mutex> lock(mu);
+    auto it = cache.find(name);
+    if (it != cache.end()) return it->second;
+    const char* v = getenv(name);
+    int r = v ? atoi(v) : dflt;
+    cache[name] = r;
+    return r;
+}
+
 // resident blocks per SM of a kernel (cached per function / block / smem)
 int occupancy(const void* fn, int threads, size_t smem) {
     static std::mutex mu;
@@ -847,6 +873,7 @@ extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, 
             mine = (mine + opts.shard_count - 1) / opts.shard_count;
             grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy(kernel_for(1, npc), 256, 0),
                                                           (mine + 7) / 8));
+            if (tune("FSGC_EDGE_BLOCKS", 0) > 0) grid = tune("FSGC_EDGE_BLOCKS", 0);
         } else {
             smem = (size_t)kWarps * 33 * (1u << cp.q) * sizeof(uint32_t);
             int64_t nchunks = ((e - b) + W.chunk - 1) / W.chunk;
@@ -868,7 +895,7 @@ extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, 
         unsigned long long* dqueue2 = dmatch + 2;
         unsigned int* dticket = (unsigned int*)(dmatch + 3);
         int* dsup = (int*)(scratch.ptr + sup_off);
-        Sink S{dacc, dmatch, (BlockPartial*)(scratch.ptr + parts_off), dticket};
+        Sink S{dacc, dmatch, (BlockPartial*)(scratch.ptr + parts_off), dticket, tune("FSGC_PUBLISH", 0)};
 
         static thread_local cudaEvent_t ev0 = nullptr, ev1 = nullptr, ev2 = nullptr;
         if (!ev0) {
