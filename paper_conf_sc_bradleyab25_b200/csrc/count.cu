@@ -27,6 +27,7 @@
 #include <tuple>
 #include <string>
 #include <cstdlib>
+#include <cstdio>
 #include "devbuf.cuh"
 #include "u128.cuh"
 #include "fc.cuh"
@@ -48,7 +49,14 @@ struct WorkDesc {
     int32_t shard, nshards;
     int32_t chunk;        // items per queue grab
     int32_t degfilter;    // 1: apply the degree filter
+    unsigned long long* trace;  // optional per-warp (start, end, smid, chunks) timing
 };
+
+__device__ __forceinline__ unsigned long long gtimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
 
 struct AccDev {
     unsigned long long lo, hi;
@@ -468,9 +476,12 @@ __global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, c
     const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const bool oriented = P.root_mode == ROOT_ORIENTED;
+    const unsigned long long t_start = W.trace ? gtimer() : 0;
+    int nch = 0;
     for (int64_t c0 = warp; ; c0 += nwarps) {          // chunks dealt round-robin to shards
         const int64_t g = c0 * W.nshards + W.shard;
         if (g >= nchunks) break;
+        ++nch;
         int u[kEdgeILP], v[kEdgeILP];
         int64_t e[kEdgeILP];
         bool ok[kEdgeILP];
@@ -507,6 +518,12 @@ __global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, c
                 acc.add((int)(w >> 24), f, o);
             }
         }
+    }
+    if (W.trace && lane == 0) {
+        unsigned smid;
+        asm volatile("mov.u32 %0, %smid;" : "=r"(smid));
+        unsigned long long* tr = W.trace + 4 * warp;
+        tr[0] = t_start; tr[1] = gtimer(); tr[2] = smid; tr[3] = (unsigned long long)nch;
     }
     block_publish<NP>(acc, nmatch, S);
 }
@@ -853,7 +870,7 @@ extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, 
         GraphDev G{g->offsets, g->adj, g->row, g->osrc, g->odst};
         OrientDev O{g->split, g->oofs};
         WorkDesc W{b, e, opts.shard_index, opts.shard_count, 4,
-                   (opts.flags & FSGC_FLAG_NO_DEGREE_FILTER) ? 0 : 1};
+                   (opts.flags & FSGC_FLAG_NO_DEGREE_FILTER) ? 0 : 1, nullptr};
         const int nsm = sm_count();
         const int npc = np_class(npm);
 
@@ -911,6 +928,12 @@ extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, 
             ++launches;
         }
         FSGC_CUDA(cudaEventRecord(ev1, st));
+        DevBuf<unsigned long long> trace;
+        if (tune("FSGC_TRACE", 0) && edge) {
+            FSGC_CUDA(trace.alloc((size_t)grid * 8 * 4, st));
+            FSGC_CUDA(cudaMemsetAsync(trace.ptr, 0, (size_t)grid * 8 * 4 * 8, st));
+            W.trace = trace.ptr;
+        }
         if (e > b) {
             ++launches;
             const int kind = cp.root_mode == ROOT_VERTEX ? 0 : edge ? 1 : 2;
@@ -934,6 +957,26 @@ extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, 
         const AccDev* hacc = host.acc;
         const unsigned long long hmatch = host.match;
         FSGC_CUDA(cudaStreamSynchronize(st));
+        if (W.trace) {
+            std::vector<unsigned long long> h((size_t)grid * 8 * 4);
+            FSGC_CUDA(cudaMemcpy(h.data(), W.trace, h.size() * 8, cudaMemcpyDeviceToHost));
+            unsigned long long t0 = ~0ull, t1 = 0;
+            std::vector<std::pair<unsigned long long, int>> d;
+            for (size_t w = 0; w < h.size() / 4; ++w) {
+                if (!h[4 * w]) continue;
+                t0 = std::min(t0, h[4 * w]);
+                t1 = std::max(t1, h[4 * w + 1]);
+                d.push_back({h[4 * w + 1] - h[4 * w], (int)w});
+            }
+            std::sort(d.rbegin(), d.rend());
+            fprintf(stderr, "[trace] warps=%zu span=%.1fus; slowest:", d.size(), (t1 - t0) / 1e3);
+            for (size_t i = 0; i < std::min<size_t>(6, d.size()); ++i) {
+                int w = d[i].second;
+                fprintf(stderr, " w%d(sm%llu,ch%llu,start+%.1f,%.1fus)", w, h[4 * w + 2], h[4 * w + 3],
+                        (h[4 * w] - t0) / 1e3, d[i].first / 1e3);
+            }
+            fprintf(stderr, "\n");
+        }
         float kms = 0.f, ams = 0.f;
         FSGC_CUDA(cudaEventElapsedTime(&ams, ev0, ev1));
         FSGC_CUDA(cudaEventElapsedTime(&kms, ev1, ev2));
