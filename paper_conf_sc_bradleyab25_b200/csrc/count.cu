@@ -23,6 +23,7 @@
 #include <algorithm>
 #include <cstring>
 #include <map>
+#include <set>
 #include <mutex>
 #include <tuple>
 #include <string>
@@ -33,6 +34,24 @@
 #include "fc.cuh"
 
 #define FULLMASK 0xffffffffu
+
+// Pascal's triangle, one thread per k column walking n (mod 2^64)
+__global__ void binom_table_init() {
+    const int k = threadIdx.x;
+    if (k >= kBinomK) return;
+    // C(n, k) = C(n-1, k) + C(n-1, k-1): do it row-serially in one warp
+    __shared__ uint64_t row[kBinomK];
+    for (int n = 0; n < kBinomN; ++n) {
+        uint64_t v;
+        if (k == 0) v = 1;
+        else if (n == 0) v = 0;
+        else v = row[k] + row[k - 1];
+        __syncwarp();
+        row[k] = v;
+        g_binom[n][k] = v;
+        __syncwarp();
+    }
+}
 
 namespace {
 
@@ -471,32 +490,37 @@ __global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, c
     acc.init();
     unsigned long long nmatch = 0;
     const int64_t total = W.end - W.begin;
-    constexpr int SPAN = 32 * kEdgeILP;
-    const int64_t nchunks = (total + SPAN - 1) / SPAN;
-    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    // this shard owns the 32-item chunks g = c * nshards + shard; its items are
+    // numbered L = c * 32 + lane and walked grid-stride, kEdgeILP at a time:
+    // a lane's items lie far apart, so the heavy roots (highest ids, at the
+    // end) are spread over many lanes instead of piling up in one
+    const int64_t nchunks = (total + 31) / 32;
+    const int64_t mychunks = nchunks > W.shard ? (nchunks - W.shard + W.nshards - 1) / W.nshards : 0;
+    const int64_t nloc = mychunks * 32;
+    const int64_t nthreads = (int64_t)gridDim.x * blockDim.x;
+    const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    const int64_t warp = tid >> 5;
     const bool oriented = P.root_mode == ROOT_ORIENTED;
     const unsigned long long t_start = W.trace ? gtimer() : 0;
     int nch = 0;
-    for (int64_t c0 = warp; ; c0 += nwarps) {          // chunks dealt round-robin to shards
-        const int64_t g = c0 * W.nshards + W.shard;
-        if (g >= nchunks) break;
+    for (int64_t L0 = tid; L0 - lane < nloc; L0 += nthreads * kEdgeILP) {
         ++nch;
         int u[kEdgeILP], v[kEdgeILP];
-        int64_t e[kEdgeILP];
+        int64_t e[kEdgeILP], itm[kEdgeILP];
         bool ok[kEdgeILP];
 #pragma unroll
         for (int j = 0; j < kEdgeILP; ++j) {           // 1: root edges (coalesced)
-            const int64_t t = g * SPAN + j * 32 + lane;
-            ok[j] = t < total;
-            const int64_t item = W.begin + (ok[j] ? t : 0);
-            if (oriented) { u[j] = __ldg(G.osrc + item); v[j] = __ldg(G.odst + item); e[j] = item; }
-            else { u[j] = __ldg(G.row + item); v[j] = __ldg(G.adj + item); }
+            const int64_t L = L0 + j * nthreads;
+            const int64_t t = ((L >> 5) * W.nshards + W.shard) * 32 + (L & 31);
+            ok[j] = L < nloc && t < total;
+            itm[j] = W.begin + (ok[j] ? t : 0);
+            if (oriented) { u[j] = __ldg(G.osrc + itm[j]); v[j] = __ldg(G.odst + itm[j]); e[j] = itm[j]; }
+            else { u[j] = __ldg(G.row + itm[j]); v[j] = __ldg(G.adj + itm[j]); }
         }
         int du[kEdgeILP], dv[kEdgeILP], c[kEdgeILP];
 #pragma unroll
         for (int j = 0; j < kEdgeILP; ++j) {           // 2: degrees + support
-            if (!oriented) e[j] = edge_of_entry(G, O, u[j], v[j], W.begin + (ok[j] ? g * SPAN + j * 32 + lane : 0));
+            if (!oriented) e[j] = edge_of_entry(G, O, u[j], v[j], itm[j]);
             du[j] = (int)(__ldg(G.offs + u[j] + 1) - __ldg(G.offs + u[j]));
             dv[j] = (int)(__ldg(G.offs + v[j] + 1) - __ldg(G.offs + v[j]));
             c[j] = __ldg(sup + e[j]);
@@ -815,6 +839,19 @@ extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, 
         FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_count: bad shard %d/%d", opts.shard_index, opts.shard_count);
     cudaStream_t st = (cudaStream_t)stream_;
     std::memset(results, 0, sizeof(fsgc_result) * npats);
+    {   // binomial table, once per device
+        static std::mutex mu;
+        static std::set<int> ready;
+        int dev = 0;
+        FSGC_CUDA(cudaGetDevice(&dev));
+        std::lock_guard<std::mutex> lock(mu);
+        if (!ready.count(dev)) {
+            binom_table_init<<<1, 32, 0, st>>>();
+            FSGC_CUDA(cudaGetLastError());
+            FSGC_CUDA(cudaStreamSynchronize(st));
+            ready.insert(dev);
+        }
+    }
 
     // passes: isomorphic cores share one pass (one Venn per core match for
     // all their fringe programs) as long as the pass fits the program limits.

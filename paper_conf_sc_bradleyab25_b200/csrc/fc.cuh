@@ -16,6 +16,12 @@
 #include "internal.h"
 #include "u128.cuh"
 
+// C(n, k) for n < kBinomN, k < kBinomK, filled once per device by
+// fsgc_binom_table_init (entries that exceed 2^64 wrap; Exact64 never reads
+// them because it only runs when N^K < 2^63, hence C(n, k) < 2^63)
+constexpr int kBinomN = 2048, kBinomK = 8;
+static __device__ uint64_t g_binom[kBinomN][kBinomK];   // (fc.cuh is included by count.cu only)
+
 struct Exact64 {
     typedef uint64_t T;
     static constexpr bool is_wide = false;
@@ -25,6 +31,7 @@ struct Exact64 {
         if (k > n) return 0;
         if (k == 0) return 1;
         if (k == 1) return n;
+        if (n < (uint64_t)kBinomN && k < (uint32_t)kBinomK) return __ldg(&g_binom[n][k]);
         if (k == 2) return (n & 1) ? n * ((n - 1) >> 1) : (n >> 1) * (n - 1);
         uint64_t r = 1;
         for (uint32_t i = 1; i <= k; ++i) r = exact_div(r * (n - k + i), i);
