@@ -255,16 +255,37 @@ def main():
     probe = F.fsgc_count(g, cps, no_degree_filter=True, shard_index=0, shard_count=1)
     core_matches = sum(r.core_matches for r in probe)
 
-    def step():
-        if world > 1:
-            return F.fsgc_count_distributed(g, cps)
-        return F.fsgc_count(g, cps)
-
     stream = torch.cuda.current_stream()
+    if world > 1:
+        def step():
+            return F.fsgc_count_distributed(g, cps)
+        replay = None
+    else:
+        # one CUDA graph per step: workspace zeroing, every kernel of every
+        # pass, and the copy of the raw 128-bit results into pinned memory
+        plan = F.fsgc_plan_create(g, cps)
+        side = torch.cuda.Stream()
+        side.wait_stream(stream)
+        with torch.cuda.stream(side):
+            plan.enqueue(side)
+        side.synchronize()
+        cg = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(cg):
+            plan.enqueue(torch.cuda.current_stream())
+        torch.cuda.synchronize()
+
+        def step():
+            cg.replay()
+            torch.cuda.current_stream().synchronize()
+            return plan.decode()
+        replay = cg
+
     flush = torch.empty(64 * 1024 * 1024, dtype=torch.int32, device=dev)   # 256 MiB > 126 MB L2
     for _ in range(args.warmup):
         res = step()
     counts = [r.count for r in res]
+    ref = F.fsgc_count(g, cps)                       # the synchronous API agrees
+    assert [r.count for r in ref] == counts, (counts, [r.count for r in ref])
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
@@ -280,10 +301,18 @@ def main():
         torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
-        ev0[s].record(stream)
-        res = step()
-        ev1[s].record(stream)
-        torch.cuda.synchronize()
+        if replay is not None:
+            ev0[s].record(stream)
+            replay.replay()
+            ev1[s].record(stream)
+            torch.cuda.synchronize()
+            res = plan.decode()
+        else:
+            ev0[s].record(stream)
+            res = step()
+            ev1[s].record(stream)
+            torch.cuda.synchronize()
+        assert [r.count for r in res] == counts
         kms.append(res[0].kernel_ms)
         ams.append(res[0].aux_ms)
         launches += res[0].kernel_launches

@@ -34,6 +34,7 @@
 #ifndef FSGC_H
 #define FSGC_H
 
+#include <stddef.h>
 #include <stdint.h>
 
 #ifdef __cplusplus
@@ -226,6 +227,37 @@ int fsgc_num_roots(const fsgc_graph* g, const fsgc_pattern* p,
  * where divisor is taken from a result of the same pattern and mode. */
 int fsgc_finalize(fsgc_u128 raw, uint64_t divisor, int32_t overflow,
                   fsgc_u128* count, int32_t* count_overflow);
+
+/* ------------------------------------------------------------- plans */
+/*
+ * Reusable, CUDA-graph-capturable execution of fsgc_count.
+ *
+ *   fsgc_plan_create      host: group the patterns into passes, build the
+ *                         fringe programs, size the grids and the workspace
+ *                         (initialises the device binomial table once per
+ *                         device, synchronously).  The plan keeps pointers to
+ *                         `g` and must not outlive it.
+ *   fsgc_plan_workspace_bytes  device workspace size (*ws) and raw result
+ *                         block size (*raw) the plan needs
+ *   fsgc_plan_enqueue     stream-ordered: zero the workspace header, run
+ *                         every pass's kernels, copy the raw 128-bit sums and
+ *                         flags to `raw_out` (device or pinned host memory,
+ *                         *raw bytes).  No allocation and no host
+ *                         synchronisation, so it can be captured in a CUDA
+ *                         graph.  One plan must not be enqueued concurrently
+ *                         on two streams with the same workspace.
+ *   fsgc_plan_decode      after the stream completed: raw block -> results
+ *                         (as fsgc_count returns them; kernel_ms / aux_ms are
+ *                         best effort, -1 when unavailable)
+ */
+typedef struct fsgc_plan fsgc_plan;
+
+int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* pats, int npats,
+                     const fsgc_count_opts* opts, fsgc_plan** out);
+int fsgc_plan_workspace_bytes(const fsgc_plan* plan, size_t* ws, size_t* raw);
+int fsgc_plan_enqueue(const fsgc_plan* plan, void* workspace, void* raw_out, void* stream);
+int fsgc_plan_decode(const fsgc_plan* plan, const void* raw, fsgc_result* results);
+void fsgc_plan_free(fsgc_plan* plan);
 
 /* thread-local message for the last failing call ("" if none) */
 const char* fsgc_last_error(void);

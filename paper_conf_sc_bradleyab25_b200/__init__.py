@@ -8,6 +8,7 @@ from ._lib import FsgcError, LIB_PATH, EXPORTS  # noqa: F401
 from .api import (  # noqa: F401
     Graph, Pattern, CountResult, fsgc_load_graph, fsgc_compile_pattern, compile_named,
     fsgc_count, fsgc_count_distributed, combine_partials, fsgc_num_roots, fsgc_finalize,
+    Plan, fsgc_plan_create,
 )
 
 __all__ = [

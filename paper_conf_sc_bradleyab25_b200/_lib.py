@@ -26,6 +26,8 @@ EXPORTS = [
     "fsgc_load_graph", "fsgc_graph_get_info", "fsgc_graph_download", "fsgc_free_graph",
     "fsgc_compile_pattern", "fsgc_pattern_get_info", "fsgc_free_pattern",
     "fsgc_count", "fsgc_num_roots", "fsgc_finalize", "fsgc_last_error", "fsgc_version",
+    "fsgc_plan_create", "fsgc_plan_workspace_bytes", "fsgc_plan_enqueue", "fsgc_plan_decode",
+    "fsgc_plan_free",
 ]
 
 
@@ -84,7 +86,7 @@ class CountOpts(C.Structure):
 def _load():
     if not os.path.exists(LIB_PATH):
         raise ImportError(
-            f"{LIB_PATH} is missing: build it with `python -m paper_conf_sc_bradleyab25_b200.build` "
+            f"{LIB_PATH} is missing: build it with `python paper_conf_sc_bradleyab25_b200/build.py` "
             "(there is no CPU fallback)")
     lib = C.CDLL(LIB_PATH)
     vp, i64, i32 = C.c_void_p, C.c_int64, C.c_int32
@@ -99,6 +101,11 @@ def _load():
         "fsgc_count": ([vp, vp, C.c_int, C.POINTER(CountOpts), C.POINTER(Result), vp], C.c_int),
         "fsgc_num_roots": ([vp, vp, C.c_int, C.POINTER(i64)], C.c_int),
         "fsgc_finalize": ([u128, C.c_uint64, i32, C.POINTER(u128), C.POINTER(i32)], C.c_int),
+        "fsgc_plan_create": ([vp, vp, C.c_int, C.POINTER(CountOpts), C.POINTER(vp)], C.c_int),
+        "fsgc_plan_workspace_bytes": ([vp, C.POINTER(C.c_size_t), C.POINTER(C.c_size_t)], C.c_int),
+        "fsgc_plan_enqueue": ([vp, vp, vp, vp], C.c_int),
+        "fsgc_plan_decode": ([vp, vp, C.POINTER(Result)], C.c_int),
+        "fsgc_plan_free": ([vp], None),
         "fsgc_last_error": ([], C.c_char_p),
         "fsgc_version": ([], C.c_char_p),
     }

@@ -179,7 +179,10 @@ def fsgc_count(graph: Graph, patterns: Sequence[Pattern], stream=None, **kw) -> 
     res = (Result * len(pats))()
     o = _opts(**kw)
     check(lib.fsgc_count(graph.handle, arr, len(pats), C.byref(o), res, _stream_handle(stream)))
-    whole = o.shard_count == 1 and o.root_begin <= 0 and o.root_end < 0
+    return _results(res, o.shard_count == 1 and o.root_begin <= 0 and o.root_end < 0)
+
+
+def _results(res, whole):
     out = []
     for r in res:
         out.append(CountResult(
@@ -188,6 +191,56 @@ def fsgc_count(graph: Graph, patterns: Sequence[Pattern], stream=None, **kw) -> 
             root_pattern_vertex=r.root_pattern_vertex, kernel_ms=r.kernel_ms, aux_ms=r.aux_ms,
             kernel_launches=r.kernel_launches))
     return out
+
+
+class Plan:
+    """fsgc_plan: a reusable, CUDA-graph-capturable count.
+
+        plan = fsgc_plan_create(g, pats)
+        plan.enqueue(stream)          # async; capturable
+        torch.cuda.synchronize()
+        results = plan.decode()
+    The plan owns its device workspace and a pinned host result block."""
+
+    def __init__(self, graph, patterns, **kw):
+        import torch
+        self.graph = graph
+        self.patterns = list(patterns)
+        arr = (C.c_void_p * len(self.patterns))(*[p.handle.value for p in self.patterns])
+        self._opts = _opts(**kw)
+        self.whole = self._opts.shard_count == 1 and self._opts.root_begin <= 0 and self._opts.root_end < 0
+        h = C.c_void_p()
+        check(lib.fsgc_plan_create(graph.handle, arr, len(self.patterns), C.byref(self._opts), C.byref(h)))
+        self._h = h
+        ws, raw = C.c_size_t(), C.c_size_t()
+        check(lib.fsgc_plan_workspace_bytes(self._h, C.byref(ws), C.byref(raw)))
+        self.workspace = torch.empty(max(ws.value, 1), dtype=torch.uint8, device="cuda")
+        self.raw = torch.empty(max(raw.value, 1), dtype=torch.uint8).pin_memory()
+        self.workspace_bytes, self.raw_bytes = ws.value, raw.value
+
+    def enqueue(self, stream=None):
+        check(lib.fsgc_plan_enqueue(self._h, C.c_void_p(self.workspace.data_ptr()),
+                                    C.c_void_p(self.raw.data_ptr()), _stream_handle(stream)))
+
+    def decode(self) -> List[CountResult]:
+        res = (Result * len(self.patterns))()
+        check(lib.fsgc_plan_decode(self._h, C.c_void_p(self.raw.data_ptr()), res))
+        return _results(res, self.whole)
+
+    def free(self):
+        if getattr(self, "_h", None):
+            lib.fsgc_plan_free(self._h)
+            self._h = C.c_void_p(0)
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def fsgc_plan_create(graph: Graph, patterns: Sequence[Pattern], **kw) -> Plan:
+    return Plan(graph, patterns, **kw)
 
 
 def fsgc_num_roots(graph: Graph, pattern: Pattern, no_symmetry_breaking=False) -> int:

@@ -1,7 +1,8 @@
 """Build ``libfsgc.so`` (the C-ABI library) in-tree with nvcc for sm_100a.
 
-    python -m paper_conf_sc_bradleyab25_b200.build          # incremental
-    python -m paper_conf_sc_bradleyab25_b200.build --force
+    python paper_conf_sc_bradleyab25_b200/build.py          # incremental
+    python paper_conf_sc_bradleyab25_b200/build.py --force
+(run as a script: importing the package would try to load the library)
 
 Objects go to ``paper_conf_sc_bradleyab25_b200/_build/``; the shared library to
 ``paper_conf_sc_bradleyab25_b200/libfsgc.so`` (git-ignored, travels to the GPU

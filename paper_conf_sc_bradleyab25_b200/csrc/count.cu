@@ -23,6 +23,7 @@
 #include <algorithm>
 #include <cstring>
 #include <map>
+#include <memory>
 #include <set>
 #include <mutex>
 #include <tuple>
@@ -827,176 +828,252 @@ extern "C" int fsgc_num_roots(const fsgc_graph* g, const fsgc_pattern* p, int no
     return FSGC_OK;
 }
 
-extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, int npats,
-                          const fsgc_count_opts* opts_in, fsgc_result* results, void* stream_) {
-    if (!g || !pats || !results || npats < 1 || npats > FSGC_MAX_BATCH)
-        FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_count: bad arguments");
+// pattern-only pass plans (groups, fringe programs), cached by pattern uid
+static int pass_plans(const fsgc_pattern* const* pats, int npats, int nosym, std::vector<PassPlan>* out) {
+    std::vector<uint64_t> key;
+    for (int i = 0; i < npats; ++i) key.push_back(pats[i]->uid);
+    key.push_back(nosym ? 1 : 0);
+    static std::mutex mu;
+    static std::map<std::vector<uint64_t>, std::vector<PassPlan>> cache;
+    std::lock_guard<std::mutex> lock(mu);
+    auto it = cache.find(key);
+    if (it != cache.end()) { *out = it->second; return FSGC_OK; }
+    std::vector<std::vector<int>> passes;
+    for (auto& grp : group_patterns(pats, npats)) {
+        std::vector<int> cur;
+        for (int idx : grp) {
+            std::vector<int> trial = cur;
+            trial.push_back(idx);
+            PassPlan probe;
+            if (!cur.empty() && fsgc_build_pass(pats, trial, nosym, &probe) != FSGC_OK) {
+                passes.push_back(cur);
+                cur = {idx};
+            } else {
+                cur = trial;
+            }
+        }
+        if (!cur.empty()) passes.push_back(cur);
+    }
+    std::vector<PassPlan> plans;
+    for (auto& members : passes) {
+        PassPlan plan;
+        int rc = fsgc_build_pass(pats, members, nosym, &plan);
+        if (rc) return rc;
+        plans.push_back(plan);
+    }
+    if (cache.size() > 1024) cache.clear();
+    cache[key] = plans;
+    *out = plans;
+    return FSGC_OK;
+}
+
+// binomial table, once per device (host-synchronous; done at plan creation so
+// that enqueue stays capturable)
+static int ensure_binom_table(int dev) {
+    static std::mutex mu;
+    static std::set<int> ready;
+    std::lock_guard<std::mutex> lock(mu);
+    if (ready.count(dev)) return FSGC_OK;
+    binom_table_init<<<1, 32>>>();
+    FSGC_CUDA(cudaGetLastError());
+    FSGC_CUDA(cudaDeviceSynchronize());
+    ready.insert(dev);
+    return FSGC_OK;
+}
+
+namespace {
+constexpr size_t kRawPassBytes = sizeof(AccDev) * FSGC_MAXPATS + 16;   // acc[16] | matches | pad
+constexpr size_t kHdrBytes = 1024;                                      // acc | counters
+
+struct PassExec {
+    PassPlan plan;
+    int kind = 0;              // 0 vertex, 1 edge (support + fc), 2 general core
+    int npc = 1;               // accumulator width class
+    int64_t grid = 1, grid_sup = 1;
+    size_t smem = 0;
+    WorkDesc W{};
+    size_t ws_off = 0, sup_bytes = 0, parts_off = 0, bytes = 0;
+    bool whole = true;
+};
+}  // namespace
+
+struct fsgc_plan {
+    const fsgc_graph* g = nullptr;
+    int npats = 0;
+    std::vector<PassExec> passes;
+    size_t ws_bytes = 0;
+    int publish_mode = 1;
+    int device = 0;
+    std::vector<cudaEvent_t> ev;   // 3 per pass
+    unsigned long long* trace = nullptr;
+    ~fsgc_plan() {
+        for (auto e : ev) cudaEventDestroy(e);
+        if (trace) cudaFree(trace);
+    }
+};
+
+extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* pats, int npats,
+                                const fsgc_count_opts* opts_in, fsgc_plan** out) {
+    if (!out) FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_plan_create: out is NULL");
+    *out = nullptr;
+    if (!g || !pats || npats < 1 || npats > FSGC_MAX_BATCH)
+        FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_plan_create: bad arguments");
     for (int i = 0; i < npats; ++i)
-        if (!pats[i]) FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_count: null pattern %d", i);
+        if (!pats[i]) FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_plan_create: null pattern %d", i);
     fsgc_count_opts opts{0, -1, 0, 1, 0, 0};
     if (opts_in) opts = *opts_in;
     if (opts.shard_count < 1 || opts.shard_index < 0 || opts.shard_index >= opts.shard_count)
-        FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_count: bad shard %d/%d", opts.shard_index, opts.shard_count);
-    cudaStream_t st = (cudaStream_t)stream_;
-    std::memset(results, 0, sizeof(fsgc_result) * npats);
-    {   // binomial table, once per device
-        static std::mutex mu;
-        static std::set<int> ready;
-        int dev = 0;
-        FSGC_CUDA(cudaGetDevice(&dev));
-        std::lock_guard<std::mutex> lock(mu);
-        if (!ready.count(dev)) {
-            binom_table_init<<<1, 32, 0, st>>>();
-            FSGC_CUDA(cudaGetLastError());
-            FSGC_CUDA(cudaStreamSynchronize(st));
-            ready.insert(dev);
-        }
-    }
-
-    // passes: isomorphic cores share one pass (one Venn per core match for
-    // all their fringe programs) as long as the pass fits the program limits.
-    // Plans depend only on the patterns and the mode: cached by pattern uid.
-    std::vector<uint64_t> key;
-    for (int i = 0; i < npats; ++i) key.push_back(pats[i]->uid);
-    key.push_back(opts.no_symmetry_breaking ? 1 : 0);
+        FSGC_FAIL(FSGC_ERR_INVALID, "bad shard %d/%d", opts.shard_index, opts.shard_count);
+    int dev = 0;
+    FSGC_CUDA(cudaGetDevice(&dev));
+    int rc = ensure_binom_table(dev);
+    if (rc) return rc;
     std::vector<PassPlan> plans;
-    {
-        static std::mutex mu;
-        static std::map<std::vector<uint64_t>, std::vector<PassPlan>> cache;
-        std::lock_guard<std::mutex> lock(mu);
-        auto it = cache.find(key);
-        if (it != cache.end()) {
-            plans = it->second;
-        } else {
-            std::vector<std::vector<int>> passes;
-            for (auto& grp : group_patterns(pats, npats)) {
-                std::vector<int> cur;
-                for (int idx : grp) {
-                    std::vector<int> trial = cur;
-                    trial.push_back(idx);
-                    PassPlan probe;
-                    if (!cur.empty() && fsgc_build_pass(pats, trial, opts.no_symmetry_breaking, &probe) != FSGC_OK) {
-                        passes.push_back(cur);
-                        cur = {idx};
-                    } else {
-                        cur = trial;
-                    }
-                }
-                if (!cur.empty()) passes.push_back(cur);
-            }
-            for (auto& members : passes) {
-                PassPlan plan;
-                int rc = fsgc_build_pass(pats, members, opts.no_symmetry_breaking, &plan);
-                if (rc) return rc;
-                plans.push_back(plan);
-            }
-            if (cache.size() > 1024) cache.clear();
-            cache[key] = plans;
-        }
-    }
-    for (const PassPlan& plan : plans) {
-        const std::vector<int>& members = plan.members;
-        int rc = FSGC_OK;
-        const CoreProg& cp = plan.prog;
+    rc = pass_plans(pats, npats, opts.no_symmetry_breaking, &plans);
+    if (rc) return rc;
+
+    std::unique_ptr<fsgc_plan> P(new fsgc_plan);
+    P->g = g;
+    P->npats = npats;
+    P->device = dev;
+    P->publish_mode = tune("FSGC_PUBLISH", 1);
+    const int nsm = sm_count();
+    size_t off = 0;
+    for (const PassPlan& pp : plans) {
+        PassExec X;
+        X.plan = pp;
+        const CoreProg& cp = pp.prog;
         const int64_t R = roots_for(g, cp.root_mode);
         int64_t b = opts.root_begin < 0 ? 0 : opts.root_begin;
         int64_t e = (opts.root_end < 0 || opts.root_end > R) ? R : opts.root_end;
         if (b > e) b = e;
-
-        const int npm = (int)members.size();
-        GraphDev G{g->offsets, g->adj, g->row, g->osrc, g->odst};
-        OrientDev O{g->split, g->oofs};
-        WorkDesc W{b, e, opts.shard_index, opts.shard_count, 4,
-                   (opts.flags & FSGC_FLAG_NO_DEGREE_FILTER) ? 0 : 1, nullptr};
-        const int nsm = sm_count();
-        const int npc = np_class(npm);
-
-        // grids
-        int64_t grid = 1, grid_sup = 1;
-        size_t smem = 0;
-        const bool edge = cp.root_mode != ROOT_VERTEX && cp.p == 2;
-        if (cp.root_mode == ROOT_VERTEX) {
-            W.chunk = 256;
+        X.whole = opts.shard_count == 1 && opts.root_begin <= 0 && opts.root_end < 0;
+        X.npc = np_class((int)pp.members.size());
+        X.W = WorkDesc{b, e, opts.shard_index, opts.shard_count, 4,
+                       (opts.flags & FSGC_FLAG_NO_DEGREE_FILTER) ? 0 : 1, nullptr};
+        X.kind = cp.root_mode == ROOT_VERTEX ? 0 : (cp.p == 2 ? 1 : 2);
+        if (X.kind == 0) {
+            X.W.chunk = 256;
             int64_t work = (e - b + opts.shard_count - 1) / opts.shard_count;
-            grid = std::max<int64_t>(1, std::min<int64_t>((work + 255) / 256,
-                                                          (int64_t)nsm * occupancy(kernel_for(0, npc), 256, 0)));
-        } else if (edge) {
-            grid_sup = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy((const void*)support_kernel, 256, 0),
-                                                              (g->m + 255) / 256));
+            X.grid = std::max<int64_t>(1, std::min<int64_t>((work + 255) / 256,
+                                                            (int64_t)nsm * occupancy(kernel_for(0, X.npc), 256, 0)));
+        } else if (X.kind == 1) {
+            X.grid_sup = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy((const void*)support_kernel, 256, 0),
+                                                                (g->m + 255) / 256));
             int64_t mine = ((e - b) + 31) / 32;
             mine = (mine + opts.shard_count - 1) / opts.shard_count;
-            grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy(kernel_for(1, npc), 256, 0),
-                                                          (mine + 7) / 8));
-            if (tune("FSGC_EDGE_BLOCKS", 0) > 0) grid = tune("FSGC_EDGE_BLOCKS", 0);
+            X.grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy(kernel_for(1, X.npc), 256, 0),
+                                                            (mine + 7) / 8));
+            if (tune("FSGC_EDGE_BLOCKS", 0) > 0) X.grid = tune("FSGC_EDGE_BLOCKS", 0);
+            X.sup_bytes = (size_t)std::max<int64_t>(g->m, 1) * sizeof(int);
         } else {
-            smem = (size_t)kWarps * 33 * (1u << cp.q) * sizeof(uint32_t);
-            int64_t nchunks = ((e - b) + W.chunk - 1) / W.chunk;
+            X.smem = (size_t)kWarps * 33 * (1u << cp.q) * sizeof(uint32_t);
+            int64_t nchunks = ((e - b) + X.W.chunk - 1) / X.W.chunk;
             int64_t mine = (nchunks + opts.shard_count - 1) / opts.shard_count;
-            grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy(kernel_for(2, npc), kWarps * 32, smem),
-                                                          (mine + kWarps - 1) / kWarps));
+            X.grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy(kernel_for(2, X.npc), kWarps * 32, X.smem),
+                                                            (mine + kWarps - 1) / kWarps));
         }
+        X.parts_off = (kHdrBytes + X.sup_bytes + 255) & ~(size_t)255;
+        X.bytes = (X.parts_off + (size_t)X.grid * sizeof(BlockPartial) + 255) & ~(size_t)255;
+        X.ws_off = off;
+        off += X.bytes;
+        P->passes.push_back(X);
+    }
+    P->ws_bytes = off;
+    P->ev.resize(3 * P->passes.size());
+    for (auto& ev : P->ev) FSGC_CUDA(cudaEventCreate(&ev));
+    if (tune("FSGC_TRACE", 0)) {
+        FSGC_CUDA(cudaMalloc(&P->trace, (size_t)2 * 1024 * 1024));
+        FSGC_CUDA(cudaMemset(P->trace, 0, (size_t)2 * 1024 * 1024));
+    }
+    *out = P.release();
+    return FSGC_OK;
+}
 
-        // one scratch allocation: header | support (edge cores) | block partials
-        const size_t hdr = 1024;
-        const size_t sup_bytes = edge ? (size_t)std::max<int64_t>(g->m, 1) * sizeof(int) : 0;
-        const size_t sup_off = hdr, parts_off = (hdr + sup_bytes + 255) & ~(size_t)255;
-        DevBuf<unsigned char> scratch;
-        FSGC_CUDA(scratch.alloc(parts_off + (size_t)grid * sizeof(BlockPartial), st));
-        FSGC_CUDA(cudaMemsetAsync(scratch.ptr, 0, hdr + sup_bytes, st));
-        AccDev* dacc = (AccDev*)scratch.ptr;                               // 16 x 32 B
-        unsigned long long* dmatch = (unsigned long long*)(scratch.ptr + 512);
+extern "C" int fsgc_plan_workspace_bytes(const fsgc_plan* P, size_t* ws, size_t* raw) {
+    if (!P) FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_plan_workspace_bytes: null plan");
+    if (ws) *ws = P->ws_bytes;
+    if (raw) *raw = kRawPassBytes * P->passes.size();
+    return FSGC_OK;
+}
+
+extern "C" int fsgc_plan_enqueue(const fsgc_plan* P, void* workspace, void* raw_out, void* stream_) {
+    if (!P || !workspace || !raw_out) FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_plan_enqueue: null argument");
+    cudaStream_t st = (cudaStream_t)stream_;
+    const fsgc_graph* g = P->g;
+    GraphDev G{g->offsets, g->adj, g->row, g->osrc, g->odst};
+    OrientDev O{g->split, g->oofs};
+    for (size_t pi = 0; pi < P->passes.size(); ++pi) {
+        const PassExec& X = P->passes[pi];
+        unsigned char* base = (unsigned char*)workspace + X.ws_off;
+        FSGC_CUDA(cudaMemsetAsync(base, 0, kHdrBytes + X.sup_bytes, st));
+        AccDev* dacc = (AccDev*)base;
+        unsigned long long* dmatch = (unsigned long long*)(base + sizeof(AccDev) * FSGC_MAXPATS);
         unsigned long long* dqueue = dmatch + 1;
         unsigned long long* dqueue2 = dmatch + 2;
         unsigned int* dticket = (unsigned int*)(dmatch + 3);
-        int* dsup = (int*)(scratch.ptr + sup_off);
-        Sink S{dacc, dmatch, (BlockPartial*)(scratch.ptr + parts_off), dticket, tune("FSGC_PUBLISH", 0)};
-
-        static thread_local cudaEvent_t ev0 = nullptr, ev1 = nullptr, ev2 = nullptr;
-        if (!ev0) {
-            FSGC_CUDA(cudaEventCreate(&ev0));
-            FSGC_CUDA(cudaEventCreate(&ev1));
-            FSGC_CUDA(cudaEventCreate(&ev2));
-        }
-        int launches = 0;
-        FSGC_CUDA(cudaEventRecord(ev0, st));
-        if (edge && g->m > 0) {   // (A) per-edge common-neighbour counts (all edges)
-            support_kernel<<<(int)grid_sup, 256, 0, st>>>(G, O, g->m, dsup, dqueue2);
+        int* dsup = (int*)(base + kHdrBytes);
+        Sink S{dacc, dmatch, (BlockPartial*)(base + X.parts_off), dticket, P->publish_mode};
+        WorkDesc W = X.W;
+        if (P->trace && X.kind == 1) W.trace = P->trace;
+        const CoreProg& cp = X.plan.prog;
+        FSGC_CUDA(cudaEventRecord(P->ev[3 * pi], st));
+        if (X.kind == 1 && g->m > 0) {   // (A) per-edge common-neighbour counts (all edges)
+            support_kernel<<<(int)X.grid_sup, 256, 0, st>>>(G, O, g->m, dsup, dqueue2);
             FSGC_CUDA(cudaGetLastError());
-            ++launches;
         }
-        FSGC_CUDA(cudaEventRecord(ev1, st));
-        DevBuf<unsigned long long> trace;
-        if (tune("FSGC_TRACE", 0) && edge) {
-            FSGC_CUDA(trace.alloc((size_t)grid * 8 * 4, st));
-            FSGC_CUDA(cudaMemsetAsync(trace.ptr, 0, (size_t)grid * 8 * 4 * 8, st));
-            W.trace = trace.ptr;
-        }
-        if (e > b) {
-            ++launches;
-            const int kind = cp.root_mode == ROOT_VERTEX ? 0 : edge ? 1 : 2;
-            const void* fn = kernel_for(kind, npc);
+        FSGC_CUDA(cudaEventRecord(P->ev[3 * pi + 1], st));
+        if (W.end > W.begin) {
+            const void* fn = kernel_for(X.kind, X.npc);
             void* args_v[] = {(void*)&G, (void*)&cp, (void*)&W, (void*)&S};
             void* args_e[] = {(void*)&G, (void*)&O, (void*)&cp, (void*)&W, (void*)&dsup, (void*)&S};
             void* args_c[] = {(void*)&G, (void*)&cp, (void*)&W, (void*)&S, (void*)&dqueue};
-            if (kind == 0) {
-                FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(256), args_v, 0, st));
-            } else if (kind == 1) {   // (B) fringe counts per root edge
-                FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(256), args_e, 0, st));
-            } else {
-                FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(kWarps * 32), args_c, smem, st));
-            }
-            FSGC_CUDA(cudaGetLastError());
+            if (X.kind == 0)
+                FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(256), args_v, 0, st));
+            else if (X.kind == 1)    // (B) fringe counts per root edge
+                FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(256), args_e, 0, st));
+            else
+                FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(kWarps * 32), args_c, X.smem, st));
         }
-        FSGC_CUDA(cudaEventRecord(ev2, st));
-        struct { AccDev acc[FSGC_MAXPATS]; unsigned long long match; } host;
-        static_assert(sizeof(host) == sizeof(AccDev) * FSGC_MAXPATS + 8, "layout");
-        FSGC_CUDA(cudaMemcpyAsync(&host, dacc, sizeof host, cudaMemcpyDeviceToHost, st));
-        const AccDev* hacc = host.acc;
-        const unsigned long long hmatch = host.match;
-        FSGC_CUDA(cudaStreamSynchronize(st));
-        if (W.trace) {
-            std::vector<unsigned long long> h((size_t)grid * 8 * 4);
-            FSGC_CUDA(cudaMemcpy(h.data(), W.trace, h.size() * 8, cudaMemcpyDeviceToHost));
+        FSGC_CUDA(cudaEventRecord(P->ev[3 * pi + 2], st));
+        FSGC_CUDA(cudaMemcpyAsync((unsigned char*)raw_out + pi * kRawPassBytes, base, kRawPassBytes - 8,
+                                  cudaMemcpyDefault, st));
+    }
+    return FSGC_OK;
+}
+
+extern "C" int fsgc_plan_decode(const fsgc_plan* P, const void* raw, fsgc_result* results) {
+    if (!P || !raw || !results) FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_plan_decode: null argument");
+    std::memset(results, 0, sizeof(fsgc_result) * P->npats);
+    for (size_t pi = 0; pi < P->passes.size(); ++pi) {
+        const PassExec& X = P->passes[pi];
+        const AccDev* acc = (const AccDev*)((const unsigned char*)raw + pi * kRawPassBytes);
+        unsigned long long matches;
+        std::memcpy(&matches, (const unsigned char*)raw + pi * kRawPassBytes + sizeof(AccDev) * FSGC_MAXPATS, 8);
+        float kms = 0.f, ams = 0.f;
+        if (cudaEventElapsedTime(&ams, P->ev[3 * pi], P->ev[3 * pi + 1]) != cudaSuccess) ams = -1.f;
+        if (cudaEventElapsedTime(&kms, P->ev[3 * pi + 1], P->ev[3 * pi + 2]) != cudaSuccess) kms = -1.f;
+        cudaGetLastError();   // timing is best effort (e.g. events recorded inside a graph)
+        const int launches = (X.W.end > X.W.begin ? 1 : 0) + (X.kind == 1 && P->g->m > 0 ? 1 : 0);
+        for (size_t mi = 0; mi < X.plan.members.size(); ++mi) {
+            fsgc_result& r = results[X.plan.members[mi]];
+            r.raw.lo = acc[mi].lo;
+            r.raw.hi = acc[mi].hi;
+            r.overflow = acc[mi].ovf ? 1 : 0;
+            r.divisor = X.plan.divisor[mi];
+            r.core_matches = matches;
+            r.root_pattern_vertex = X.plan.root_pattern_vertex[mi];
+            r.kernel_ms = kms;
+            r.aux_ms = ams;
+            r.kernel_launches = launches;
+            if (X.whole) {
+                int rc = fsgc_finalize(r.raw, r.divisor, r.overflow, &r.count, &r.overflow);
+                if (rc) return rc;
+            }
+        }
+        if (P->trace && X.kind == 1) {
+            std::vector<unsigned long long> h((size_t)2 * 1024 * 1024 / 8);
+            FSGC_CUDA(cudaMemcpy(h.data(), P->trace, h.size() * 8, cudaMemcpyDeviceToHost));
             unsigned long long t0 = ~0ull, t1 = 0;
             std::vector<std::pair<unsigned long long, int>> d;
             for (size_t w = 0; w < h.size() / 4; ++w) {
@@ -1014,25 +1091,80 @@ extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, 
             }
             fprintf(stderr, "\n");
         }
-        float kms = 0.f, ams = 0.f;
-        FSGC_CUDA(cudaEventElapsedTime(&ams, ev0, ev1));
-        FSGC_CUDA(cudaEventElapsedTime(&kms, ev1, ev2));
-        for (int mi = 0; mi < npm; ++mi) {
-            fsgc_result& r = results[members[mi]];
-            r.raw.lo = hacc[mi].lo;
-            r.raw.hi = hacc[mi].hi;
-            r.overflow = hacc[mi].ovf ? 1 : 0;
-            r.divisor = plan.divisor[mi];
-            r.core_matches = hmatch;
-            r.root_pattern_vertex = plan.root_pattern_vertex[mi];
-            r.kernel_ms = kms;
-            r.aux_ms = ams;
-            r.kernel_launches = launches;
-            if (opts.shard_count == 1 && opts.root_begin <= 0 && opts.root_end < 0) {
-                rc = fsgc_finalize(r.raw, r.divisor, r.overflow, &r.count, &r.overflow);
-                if (rc) return rc;
-            }
-        }
     }
     return FSGC_OK;
+}
+
+extern "C" void fsgc_plan_free(fsgc_plan* P) { delete P; }
+
+// ---------------------------------------------------------------- fsgc_count
+// Convenience path: cached plan + per-thread workspace / pinned result
+// buffers, enqueue, synchronise, decode.
+namespace {
+struct ThreadBuffers {
+    void* ws = nullptr;
+    size_t ws_size = 0;
+    int ws_dev = -1;
+    void* raw = nullptr;
+    size_t raw_size = 0;
+    ~ThreadBuffers() {
+        if (ws) cudaFree(ws);
+        if (raw) cudaFreeHost(raw);
+    }
+};
+}  // namespace
+
+extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, int npats,
+                          const fsgc_count_opts* opts_in, fsgc_result* results, void* stream_) {
+    if (!g || !pats || !results || npats < 1 || npats > FSGC_MAX_BATCH)
+        FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_count: bad arguments");
+    for (int i = 0; i < npats; ++i)
+        if (!pats[i]) FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_count: null pattern %d", i);
+    fsgc_count_opts opts{0, -1, 0, 1, 0, 0};
+    if (opts_in) opts = *opts_in;
+    cudaStream_t st = (cudaStream_t)stream_;
+
+    // plan cache: graph identity + pattern uids + options
+    std::vector<uint64_t> key{g->uid, (uint64_t)opts.root_begin, (uint64_t)opts.root_end,
+                              (uint64_t)opts.shard_index, (uint64_t)opts.shard_count,
+                              (uint64_t)opts.no_symmetry_breaking, (uint64_t)opts.flags};
+    for (int i = 0; i < npats; ++i) key.push_back(pats[i]->uid);
+    static std::mutex mu;
+    static std::map<std::vector<uint64_t>, std::shared_ptr<fsgc_plan>> cache;
+    std::shared_ptr<fsgc_plan> plan;
+    {
+        std::lock_guard<std::mutex> lock(mu);
+        auto it = cache.find(key);
+        if (it != cache.end()) plan = it->second;
+    }
+    if (!plan) {
+        fsgc_plan* p = nullptr;
+        int rc = fsgc_plan_create(g, pats, npats, &opts, &p);
+        if (rc) return rc;
+        plan.reset(p, fsgc_plan_free);
+        std::lock_guard<std::mutex> lock(mu);
+        if (cache.size() > 256) cache.clear();
+        cache[key] = plan;
+    }
+    static thread_local ThreadBuffers tb;
+    size_t wsb = 0, rawb = 0;
+    fsgc_plan_workspace_bytes(plan.get(), &wsb, &rawb);
+    if (tb.ws_size < wsb || tb.ws_dev != plan->device) {
+        if (tb.ws) cudaFree(tb.ws);
+        tb.ws = nullptr;
+        tb.ws_size = 0;
+        FSGC_CUDA(cudaMalloc(&tb.ws, std::max<size_t>(wsb, 1 << 20)));
+        tb.ws_size = std::max<size_t>(wsb, 1 << 20);
+        tb.ws_dev = plan->device;
+    }
+    if (tb.raw_size < rawb) {
+        if (tb.raw) cudaFreeHost(tb.raw);
+        tb.raw = nullptr;
+        FSGC_CUDA(cudaMallocHost(&tb.raw, std::max<size_t>(rawb, 4096)));
+        tb.raw_size = std::max<size_t>(rawb, 4096);
+    }
+    int rc = fsgc_plan_enqueue(plan.get(), tb.ws, tb.raw, st);
+    if (rc) return rc;
+    FSGC_CUDA(cudaStreamSynchronize(st));
+    return fsgc_plan_decode(plan.get(), tb.raw, results);
 }

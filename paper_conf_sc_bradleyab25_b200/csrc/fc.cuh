@@ -29,13 +29,26 @@ struct Exact64 {
     static __device__ __forceinline__ T mul(T a, T b, bool&) { return a * b; }
     static __device__ __forceinline__ T binom(uint64_t n, uint32_t k, bool&) {
         if (k > n) return 0;
-        if (k == 0) return 1;
-        if (k == 1) return n;
+        switch (k) {   // falling factorial / k!, exact division (no memory, no div)
+            case 0: return 1;
+            case 1: return n;
+            case 2: return (n & 1) ? n * ((n - 1) >> 1) : (n >> 1) * (n - 1);
+            case 3: return exact_div_const<6>(n * (n - 1) * (n - 2));
+            case 4: return exact_div_const<24>(n * (n - 1) * (n - 2) * (n - 3));
+            default: break;
+        }
         if (n < (uint64_t)kBinomN && k < (uint32_t)kBinomK) return __ldg(&g_binom[n][k]);
-        if (k == 2) return (n & 1) ? n * ((n - 1) >> 1) : (n >> 1) * (n - 1);
         uint64_t r = 1;
         for (uint32_t i = 1; i <= k; ++i) r = exact_div(r * (n - k + i), i);
         return r;
+    }
+    template <uint32_t D>
+    static __device__ __forceinline__ uint64_t exact_div_const(uint64_t x) {
+        constexpr int tz = __builtin_ctz(D);
+        constexpr uint64_t od = D >> tz;
+        constexpr uint64_t i0 = od, i1 = i0 * (2 - od * i0), i2 = i1 * (2 - od * i1), i3 = i2 * (2 - od * i2),
+                           i4 = i3 * (2 - od * i3), inv = i4 * (2 - od * i4);
+        return (x >> tz) * inv;
     }
     // x / d for d | x (exact): shift out the 2-adic part, multiply by the
     // inverse of the odd part mod 2^64 (Newton: 5 steps from 3 correct bits)

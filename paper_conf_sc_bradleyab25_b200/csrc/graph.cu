@@ -14,6 +14,7 @@
 // HBM layout of the result: offsets int64[n+1], adj int32[2m], row int32[2m],
 // osrc/odst int32[m] (SoA, sorted by (u, v)), order int32[n].
 #include <cub/cub.cuh>
+#include <atomic>
 #include "devbuf.cuh"
 
 namespace {
@@ -299,6 +300,8 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
     FSGC_CUDA(cudaStreamSynchronize(st));
 
     fsgc_graph* g = new fsgc_graph;
+    static std::atomic<uint64_t> next_uid{1};
+    g->uid = next_uid.fetch_add(1);
     g->n = n;
     g->m = m;
     g->max_degree = maxdeg;

@@ -17,6 +17,7 @@ void fsgc_set_error(const char* fmt, ...);
 
 // --------------------------------------------------------------- handles
 struct fsgc_graph {
+    uint64_t uid = 0;            // unique per loaded graph (plan cache key)
     int64_t n = 0, m = 0, max_degree = 0;
     int64_t* offsets = nullptr;  // [n+1]
     int32_t* adj = nullptr;      // [2m]
