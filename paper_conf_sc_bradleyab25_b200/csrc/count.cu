@@ -406,14 +406,17 @@ __device__ __forceinline__ int support_warp(const int32_t* __restrict__ adj, con
 }
 
 __global__ void __launch_bounds__(256) support_kernel(GraphDev G, OrientDev O, int64_t m, int* __restrict__ sup,
-                                                      unsigned long long* queue) {
+                                                      unsigned long long* queue, unsigned long long* trace) {
     const int lane = threadIdx.x & 31;
+    const unsigned long long t_start = trace ? gtimer() : 0;
+    int nch = 0;
     for (;;) {
         unsigned long long jq = 0;
         if (lane == 0) jq = atomicAdd(queue, 1ull);
         jq = __shfl_sync(FULLMASK, jq, 0);
         const int64_t t0 = (int64_t)jq * 32;
         if (t0 >= m) break;
+        ++nch;
         const int64_t t = t0 + lane;
         const bool valid = t < m;
         const int64_t e = valid ? m - 1 - t : 0;     // heavy (high-id) roots first
@@ -439,6 +442,12 @@ __global__ void __launch_bounds__(256) support_kernel(GraphDev G, OrientDev O, i
             if (lane == who) c = cc;
         }
         if (valid && c) atomicAdd(sup + e, c);
+    }
+    if (trace && lane == 0) {
+        unsigned smid;
+        asm volatile("mov.u32 %0, %smid;" : "=r"(smid));
+        unsigned long long* tr = trace + 4 * ((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
+        tr[0] = t_start; tr[1] = gtimer(); tr[2] = smid; tr[3] = (unsigned long long)nch;
     }
 }
 
@@ -1000,6 +1009,10 @@ extern "C" int fsgc_plan_workspace_bytes(const fsgc_plan* P, size_t* ws, size_t*
 extern "C" int fsgc_plan_enqueue(const fsgc_plan* P, void* workspace, void* raw_out, void* stream_) {
     if (!P || !workspace || !raw_out) FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_plan_enqueue: null argument");
     cudaStream_t st = (cudaStream_t)stream_;
+    cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+    FSGC_CUDA(cudaStreamIsCapturing(st, &cap));
+    // inside a graph capture the timing events must be "external" records
+    const unsigned evflags = cap == cudaStreamCaptureStatusActive ? cudaEventRecordExternal : 0;
     const fsgc_graph* g = P->g;
     GraphDev G{g->offsets, g->adj, g->row, g->osrc, g->odst};
     OrientDev O{g->split, g->oofs};
@@ -1017,12 +1030,13 @@ extern "C" int fsgc_plan_enqueue(const fsgc_plan* P, void* workspace, void* raw_
         WorkDesc W = X.W;
         if (P->trace && X.kind == 1) W.trace = P->trace;
         const CoreProg& cp = X.plan.prog;
-        FSGC_CUDA(cudaEventRecord(P->ev[3 * pi], st));
+        FSGC_CUDA(cudaEventRecordWithFlags(P->ev[3 * pi], st, evflags));
         if (X.kind == 1 && g->m > 0) {   // (A) per-edge common-neighbour counts (all edges)
-            support_kernel<<<(int)X.grid_sup, 256, 0, st>>>(G, O, g->m, dsup, dqueue2);
+            support_kernel<<<(int)X.grid_sup, 256, 0, st>>>(G, O, g->m, dsup, dqueue2,
+                                                             P->trace ? P->trace + (1 << 17) : nullptr);
             FSGC_CUDA(cudaGetLastError());
         }
-        FSGC_CUDA(cudaEventRecord(P->ev[3 * pi + 1], st));
+        FSGC_CUDA(cudaEventRecordWithFlags(P->ev[3 * pi + 1], st, evflags));
         if (W.end > W.begin) {
             const void* fn = kernel_for(X.kind, X.npc);
             void* args_v[] = {(void*)&G, (void*)&cp, (void*)&W, (void*)&S};
@@ -1035,7 +1049,7 @@ extern "C" int fsgc_plan_enqueue(const fsgc_plan* P, void* workspace, void* raw_
             else
                 FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(kWarps * 32), args_c, X.smem, st));
         }
-        FSGC_CUDA(cudaEventRecord(P->ev[3 * pi + 2], st));
+        FSGC_CUDA(cudaEventRecordWithFlags(P->ev[3 * pi + 2], st, evflags));
         FSGC_CUDA(cudaMemcpyAsync((unsigned char*)raw_out + pi * kRawPassBytes, base, kRawPassBytes - 8,
                                   cudaMemcpyDefault, st));
     }
@@ -1072,24 +1086,29 @@ extern "C" int fsgc_plan_decode(const fsgc_plan* P, const void* raw, fsgc_result
             }
         }
         if (P->trace && X.kind == 1) {
-            std::vector<unsigned long long> h((size_t)2 * 1024 * 1024 / 8);
-            FSGC_CUDA(cudaMemcpy(h.data(), P->trace, h.size() * 8, cudaMemcpyDeviceToHost));
-            unsigned long long t0 = ~0ull, t1 = 0;
-            std::vector<std::pair<unsigned long long, int>> d;
-            for (size_t w = 0; w < h.size() / 4; ++w) {
-                if (!h[4 * w]) continue;
-                t0 = std::min(t0, h[4 * w]);
-                t1 = std::max(t1, h[4 * w + 1]);
-                d.push_back({h[4 * w + 1] - h[4 * w], (int)w});
+            std::vector<unsigned long long> all((size_t)2 * 1024 * 1024 / 8);
+            FSGC_CUDA(cudaMemcpy(all.data(), P->trace, all.size() * 8, cudaMemcpyDeviceToHost));
+            for (int part = 0; part < 2; ++part) {
+                const unsigned long long* h = all.data() + (part ? (1 << 17) : 0);
+                unsigned long long t0 = ~0ull, t1 = 0;
+                std::vector<std::pair<unsigned long long, int>> d;
+                for (size_t w = 0; w < (1 << 15); ++w) {
+                    if (!h[4 * w]) continue;
+                    t0 = std::min(t0, h[4 * w]);
+                    t1 = std::max(t1, h[4 * w + 1]);
+                    d.push_back({h[4 * w + 1] - h[4 * w], (int)w});
+                }
+                std::sort(d.rbegin(), d.rend());
+                fprintf(stderr, "[trace %s] warps=%zu span=%.1fus; slowest:", part ? "support" : "fc", d.size(),
+                        (t1 - t0) / 1e3);
+                for (size_t i = 0; i < std::min<size_t>(6, d.size()); ++i) {
+                    int w = d[i].second;
+                    fprintf(stderr, " w%d(sm%llu,ch%llu,start+%.1f,%.1fus)", w, h[4 * w + 2], h[4 * w + 3],
+                            (h[4 * w] - t0) / 1e3, d[i].first / 1e3);
+                }
+                fprintf(stderr, "\n");
             }
-            std::sort(d.rbegin(), d.rend());
-            fprintf(stderr, "[trace] warps=%zu span=%.1fus; slowest:", d.size(), (t1 - t0) / 1e3);
-            for (size_t i = 0; i < std::min<size_t>(6, d.size()); ++i) {
-                int w = d[i].second;
-                fprintf(stderr, " w%d(sm%llu,ch%llu,start+%.1f,%.1fus)", w, h[4 * w + 2], h[4 * w + 3],
-                        (h[4 * w] - t0) / 1e3, d[i].first / 1e3);
-            }
-            fprintf(stderr, "\n");
+            cudaMemset(P->trace, 0, (size_t)2 * 1024 * 1024);
         }
     }
     return FSGC_OK;
