@@ -410,16 +410,16 @@ __global__ void __launch_bounds__(256) support_kernel(GraphDev G, OrientDev O, i
     const int lane = threadIdx.x & 31;
     const unsigned long long t_start = trace ? gtimer() : 0;
     int nch = 0;
-    for (;;) {
-        unsigned long long jq = 0;
-        if (lane == 0) jq = atomicAdd(queue, 1ull);
-        jq = __shfl_sync(FULLMASK, jq, 0);
-        const int64_t t0 = (int64_t)jq * 32;
-        if (t0 >= m) break;
+    const int64_t nthreads = (int64_t)gridDim.x * blockDim.x;
+    const int64_t NW = nthreads >> 5;
+    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t tpos = (int64_t)lane * NW + warp;   // transposed: hubs spread over warps
+    (void)queue;
+    for (int64_t t0 = 0; t0 < m; t0 += nthreads) {
         ++nch;
-        const int64_t t = t0 + lane;
+        const int64_t t = t0 + tpos;
         const bool valid = t < m;
-        const int64_t e = valid ? m - 1 - t : 0;     // heavy (high-id) roots first
+        const int64_t e = valid ? t : 0;
         int u = 0, v = 0, nu = 0, nv = 0;
         int64_t su = 0, sv = 0;
         if (valid) {
@@ -446,7 +446,7 @@ __global__ void __launch_bounds__(256) support_kernel(GraphDev G, OrientDev O, i
     if (trace && lane == 0) {
         unsigned smid;
         asm volatile("mov.u32 %0, %smid;" : "=r"(smid));
-        unsigned long long* tr = trace + 4 * ((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
+        unsigned long long* tr = trace + 4 * warp;
         tr[0] = t_start; tr[1] = gtimer(); tr[2] = smid; tr[3] = (unsigned long long)nch;
     }
 }
@@ -480,6 +480,7 @@ __global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, c
     // program table in shared memory: k | l << 8 | m << 16 | pattern << 24
     __shared__ uint32_t s_prog[FSGC_MAXPROG];
     __shared__ int s_kmax, s_minm;
+    __shared__ uint64_t s_venn[8][32][3];            // per warp: the roots' Venn entries
     if (threadIdx.x == 0) {
         int kmax = 0, minm = 255;
         for (int pi = 0; pi < P.nprog; ++pi) {
@@ -510,17 +511,23 @@ __global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, c
     const int64_t nthreads = (int64_t)gridDim.x * blockDim.x;
     const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     const int64_t warp = tid >> 5;
+    const int wib = threadIdx.x >> 5;
     const bool oriented = P.root_mode == ROOT_ORIENTED;
     const unsigned long long t_start = W.trace ? gtimer() : 0;
     int nch = 0;
-    for (int64_t L0 = tid; L0 - lane < nloc; L0 += nthreads * kEdgeILP) {
+    // transposed assignment: lane l of warp w takes local item l * NW + w of
+    // each NT-slice, so the hub roots (clustered at the end of the degree-
+    // ordered list) spread over all warps instead of filling a few
+    const int64_t NW = nthreads >> 5;
+    const int64_t tpos = (int64_t)lane * NW + warp;
+    for (int64_t L0 = 0; L0 < nloc; L0 += nthreads * kEdgeILP) {
         ++nch;
         int u[kEdgeILP], v[kEdgeILP];
         int64_t e[kEdgeILP], itm[kEdgeILP];
         bool ok[kEdgeILP];
 #pragma unroll
-        for (int j = 0; j < kEdgeILP; ++j) {           // 1: root edges (coalesced)
-            const int64_t L = L0 + j * nthreads;
+        for (int j = 0; j < kEdgeILP; ++j) {           // 1: root edges
+            const int64_t L = L0 + j * nthreads + tpos;
             const int64_t t = ((L >> 5) * W.nshards + W.shard) * 32 + (L & 31);
             ok[j] = L < nloc && t < total;
             itm[j] = W.begin + (ok[j] ? t : 0);
@@ -536,21 +543,37 @@ __global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, c
             c[j] = __ldg(sup + e[j]);
         }
 #pragma unroll
-        for (int j = 0; j < kEdgeILP; ++j) {           // 3: Venn + fc
-            if (!ok[j]) continue;
-            if (W.degfilter && (du[j] < P.mindeg[0] || dv[j] < P.mindeg[1])) continue;
-            ++nmatch;
-            const uint64_t cc = (uint64_t)c[j];
-            if (cc < minm) continue;                    // every program needs >= minm wedge fringes
-            const uint64_t nu = du[j] - 1 - cc, nv = dv[j] - 1 - cc;
-            const bool small = fits64(nu + nv + cc, Kmax);
-#pragma unroll 1
-            for (int pi = 0; pi < nprog; ++pi) {
+        for (int j = 0; j < kEdgeILP; ++j) {           // 3: Venn diagrams
+            bool work = false;
+            uint64_t nu = 0, nv = 0, cc = 0;
+            if (ok[j] && !(W.degfilter && (du[j] < P.mindeg[0] || dv[j] < P.mindeg[1]))) {
+                ++nmatch;
+                cc = (uint64_t)c[j];
+                work = cc >= minm;                      // every program needs >= minm wedge fringes
+                nu = du[j] - 1 - cc;
+                nv = dv[j] - 1 - cc;
+            }
+            // 4: fc over (root, program) pairs spread across the warp, so a
+            // root with a long program list does not serialise on one lane
+            const unsigned wm = __ballot_sync(FULLMASK, work);
+            if (!wm) continue;
+            if (work) {
+                s_venn[wib][lane][0] = nu;
+                s_venn[wib][lane][1] = nv;
+                s_venn[wib][lane][2] = cc;
+            }
+            __syncwarp();
+            const int total_pairs = __popc(wm) * nprog;
+            for (int t = lane; t < total_pairs; t += 32) {
+                const int k = t / nprog, pi = t - k * nprog;
+                const int src = __fns(wm, 0, k + 1);    // k-th root with work
+                const uint64_t a = s_venn[wib][src][0], b = s_venn[wib][src][1], x = s_venn[wib][src][2];
                 const uint32_t w = s_prog[pi];
                 bool o = false;
-                const u128 f = edge_prog_eval(nu, nv, cc, w, small, o);
+                const u128 f = edge_prog_eval(a, b, x, w, fits64(a + b + x, Kmax), o);
                 acc.add((int)(w >> 24), f, o);
             }
+            __syncwarp();
         }
     }
     if (W.trace && lane == 0) {
