@@ -129,15 +129,17 @@ def measured_peaks():
     return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
 
 
-def ncu_traffic(workload):
-    """dram bytes per launch of the dominant kernel from the committed ncu
-    summary (profiles/), or None."""
+def ncu_traffic(workload, kernel):
+    """dram__bytes_read + dram__bytes_write per launch of `kernel` from the
+    committed `ncu --set full` summary (profiles/ncu_summary.json), or None."""
     path = os.path.join(ROOT, "profiles", "ncu_summary.json")
     if not os.path.exists(path):
         return None
-    d = json.load(open(path))
-    w = d.get(workload)
-    return None if w is None else w.get("dram_bytes_per_launch")
+    d = json.load(open(path)).get(workload, {}).get("kernels", {})
+    for k, v in d.items():
+        if kernel.startswith(k):
+            return v.get("dram_bytes_per_launch")
+    return None
 
 
 def load_workload(name, device):
@@ -349,9 +351,8 @@ def main():
                ("support_kernel (per-edge |N(u)&N(v)| by oriented listing)", sup_bytes, aux_ms)]
     kernels.sort(key=lambda k: -k[2])
     peak, peak_src = measured_peaks()
-    traffic = ncu_traffic(args.workload)
-
-    def roof(name, byts, ms, traffic=None):
+    def roof(name, byts, ms):
+        traffic = ncu_traffic(args.workload, name)
         ach = byts / (ms / 1e3) / 1e9 if ms > 0 else 0.0
         return {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
                 "traffic": traffic, "kernel": name, "kernel_ms": ms,
@@ -409,7 +410,7 @@ def main():
                        "parallelism": f"{world} GPU(s): graph replicated, root-edge chunks dealt "
                                       f"round-robin, 1 all-reduce of 128-bit partials"},
             "gpu_launches": launches,
-            "roofline": roof(*kernels[0], traffic=traffic),
+            "roofline": roof(*kernels[0]),
             "roofline_other_kernels": [roof(*k) for k in kernels[1:]],
             "clocks": clocks,
             "e2e": e2e,

@@ -446,7 +446,7 @@ __global__ void __launch_bounds__(256) support_kernel(GraphDev G, OrientDev O, i
     if (trace && lane == 0) {
         unsigned smid;
         asm volatile("mov.u32 %0, %smid;" : "=r"(smid));
-        unsigned long long* tr = trace + 4 * warp;
+        unsigned long long* tr = trace + 8 * warp;
         tr[0] = t_start; tr[1] = gtimer(); tr[2] = smid; tr[3] = (unsigned long long)nch;
     }
 }
@@ -514,6 +514,7 @@ __global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, c
     const int wib = threadIdx.x >> 5;
     const bool oriented = P.root_mode == ROOT_ORIENTED;
     const unsigned long long t_start = W.trace ? gtimer() : 0;
+    unsigned long long tp1 = 0, tp2 = 0, tp3 = 0;
     int nch = 0;
     // transposed assignment: lane l of warp w takes local item l * NW + w of
     // each NT-slice, so the hub roots (clustered at the end of the degree-
@@ -534,6 +535,7 @@ __global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, c
             if (oriented) { u[j] = __ldg(G.osrc + itm[j]); v[j] = __ldg(G.odst + itm[j]); e[j] = itm[j]; }
             else { u[j] = __ldg(G.row + itm[j]); v[j] = __ldg(G.adj + itm[j]); }
         }
+        if (W.trace && nch == 1) { __syncwarp(); int z = u[0] + u[kEdgeILP - 1]; if (z == -7) nmatch++; tp1 = gtimer(); }
         int du[kEdgeILP], dv[kEdgeILP], c[kEdgeILP];
 #pragma unroll
         for (int j = 0; j < kEdgeILP; ++j) {           // 2: degrees + support
@@ -543,6 +545,7 @@ __global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, c
             c[j] = __ldg(sup + e[j]);
         }
 #pragma unroll
+        if (W.trace && nch == 1) { int z = c[0] + du[kEdgeILP - 1] + dv[0]; if (z == -7) nmatch++; tp2 = gtimer(); }
         for (int j = 0; j < kEdgeILP; ++j) {           // 3: Venn diagrams
             bool work = false;
             uint64_t nu = 0, nv = 0, cc = 0;
@@ -576,13 +579,15 @@ __global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, c
             __syncwarp();
         }
     }
+    tp3 = W.trace ? gtimer() : 0;
+    block_publish<NP>(acc, nmatch, S);
     if (W.trace && lane == 0) {
         unsigned smid;
         asm volatile("mov.u32 %0, %smid;" : "=r"(smid));
-        unsigned long long* tr = W.trace + 4 * warp;
+        unsigned long long* tr = W.trace + 8 * warp;
         tr[0] = t_start; tr[1] = gtimer(); tr[2] = smid; tr[3] = (unsigned long long)nch;
+        tr[4] = tp1; tr[5] = tp2; tr[6] = tp3;
     }
-    block_publish<NP>(acc, nmatch, S);
 }
 
 // ------------------------------------------------------------------------
@@ -1115,19 +1120,23 @@ extern "C" int fsgc_plan_decode(const fsgc_plan* P, const void* raw, fsgc_result
                 const unsigned long long* h = all.data() + (part ? (1 << 17) : 0);
                 unsigned long long t0 = ~0ull, t1 = 0;
                 std::vector<std::pair<unsigned long long, int>> d;
-                for (size_t w = 0; w < (1 << 15); ++w) {
-                    if (!h[4 * w]) continue;
-                    t0 = std::min(t0, h[4 * w]);
-                    t1 = std::max(t1, h[4 * w + 1]);
-                    d.push_back({h[4 * w + 1] - h[4 * w], (int)w});
+                for (size_t w = 0; w < (1 << 14); ++w) {
+                    if (!h[8 * w]) continue;
+                    t0 = std::min(t0, h[8 * w]);
+                    t1 = std::max(t1, h[8 * w + 1]);
+                    d.push_back({h[8 * w + 1] - h[8 * w], (int)w});
                 }
                 std::sort(d.rbegin(), d.rend());
                 fprintf(stderr, "[trace %s] warps=%zu span=%.1fus; slowest:", part ? "support" : "fc", d.size(),
                         (t1 - t0) / 1e3);
-                for (size_t i = 0; i < std::min<size_t>(6, d.size()); ++i) {
+                for (size_t i = 0; i < std::min<size_t>(4, d.size()); ++i) {
                     int w = d[i].second;
-                    fprintf(stderr, " w%d(sm%llu,ch%llu,start+%.1f,%.1fus)", w, h[4 * w + 2], h[4 * w + 3],
-                            (h[4 * w] - t0) / 1e3, d[i].first / 1e3);
+                    const unsigned long long* r = h + 8 * w;
+                    fprintf(stderr, " w%d(sm%llu,ch%llu,start+%.1f,%.1fus", w, r[2], r[3], (r[0] - t0) / 1e3,
+                            d[i].first / 1e3);
+                    if (r[4]) fprintf(stderr, " ld1 %.1f ld2 %.1f fc %.1f pub %.1f", (r[4] - r[0]) / 1e3,
+                                      (r[5] - r[4]) / 1e3, (r[6] - r[5]) / 1e3, (r[1] - r[6]) / 1e3);
+                    fprintf(stderr, ")");
                 }
                 fprintf(stderr, "\n");
             }
