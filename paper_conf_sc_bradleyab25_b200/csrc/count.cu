@@ -591,6 +591,239 @@ __global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, c
 }
 
 // ------------------------------------------------------------------------
+// Triangle cores (p = 3, all pairs adjacent; symmetry broken u < v < w).
+//
+// Enumeration: one lane per oriented root edge (u, v), merging the short
+// degree-oriented out-lists N+(u), N+(v): each common w is a triangle found
+// exactly once (from its lowest edge).  Lanes advance to their next match,
+// the warp ballots the lanes that found one (Listing 7) and appends those
+// core matches to a per-warp leaf buffer in shared memory.
+// Venn (Sec. 3.3): with c(xy) = |N(x) & N(y)| from the support pass and
+// t = |N(u) & N(v) & N(w)| (one triple intersection, scanning the smallest
+// list N(u) -- u has the lowest degree -- against v, w via hub bitmaps or
+// galloping cursors), the 7 regions of e(u), e(v), e(w) (core vertices
+// excluded; every core vertex is adjacent to the other two) are
+//   uvw = t, uv = c(uv)-1-t, uw = c(uw)-1-t, vw = c(vw)-1-t,
+//   u = deg(u)-2-uv-uw-t (and likewise v, w).
+// fc: Listing 5 over (leaf, program) pairs spread across the lanes.
+struct HubDev {
+    int64_t base, words;
+    const uint32_t* __restrict__ bits;
+};
+
+// galloping membership cursor over a sorted adjacency list (queries ascending)
+struct Cursor {
+    const int32_t* __restrict__ L;
+    const uint32_t* __restrict__ bm;   // hub bitmap row or nullptr
+    int len, j;
+    __device__ __forceinline__ void init(const GraphDev& G, const HubDev& H, int y) {
+        if (y >= H.base) {
+            bm = H.bits + (int64_t)(y - H.base) * H.words;
+            L = nullptr; len = 0; j = 0;
+        } else {
+            bm = nullptr;
+            const int64_t b = __ldg(G.offs + y);
+            L = G.adj + b;
+            len = (int)(__ldg(G.offs + y + 1) - b);
+            j = 0;
+        }
+    }
+    __device__ __forceinline__ bool has(int x) {
+        if (bm) return (__ldg(bm + (x >> 5)) >> (x & 31)) & 1u;
+        int lo = j;
+        if (lo >= len) return false;
+        int y = __ldg(L + lo);
+        if (y >= x) { j = lo; return y == x; }
+        int step = 1, hi = lo + 1;
+        while (hi < len && __ldg(L + hi) < x) { lo = hi; step <<= 1; hi = lo + step; }
+        if (hi > len) hi = len;
+        while (hi - lo > 1) {
+            const int mid = (lo + hi) >> 1;
+            if (__ldg(L + mid) < x) lo = mid; else hi = mid;
+        }
+        j = hi;
+        return hi < len && __ldg(L + hi) == x;
+    }
+};
+
+__device__ __forceinline__ bool member(const GraphDev& G, const HubDev& H, int y, int x) {
+    if (y >= H.base) return (__ldg(H.bits + (int64_t)(y - H.base) * H.words + (x >> 5)) >> (x & 31)) & 1u;
+    const int64_t b = __ldg(G.offs + y);
+    return contains(G.adj + b, (int)(__ldg(G.offs + y + 1) - b), x);
+}
+
+constexpr int kTriWarps = 8;
+constexpr int kTriLight = 32;     // N(u) longer than this: warp-cooperative triple intersection
+constexpr int kTriStack = 32;
+
+template <int NP>
+__global__ void __launch_bounds__(kTriWarps * 32) tri_core_kernel(GraphDev G, OrientDev O, HubDev H,
+                                                                   const CoreProg P, WorkDesc W,
+                                                                   const int* __restrict__ sup, const Sink S) {
+    __shared__ uint32_t s_leaf[kTriWarps][64][6];   // u, v, w, e(uv), e(uw), e(vw)
+    __shared__ uint32_t s_venn[kTriWarps][64][8];   // Venn over the q anchors
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    AccN<NP> acc;
+    acc.init();
+    unsigned long long nmatch = 0;
+    const int q = P.q, V = 1 << q, nprog = P.nprog;
+    // position mask F (bit0 u, bit1 v, bit2 w) -> Venn bit mask over the anchors
+    int proj[8];
+#pragma unroll
+    for (int F = 0; F < 8; ++F) {
+        int M = 0;
+        for (int b = 0; b < q; ++b)
+            if ((F >> P.anchor_pos[b]) & 1) M |= 1 << b;
+        proj[F] = M;
+    }
+    // this shard's roots, transposed over the grid (see edge_fc_kernel)
+    const int64_t total = W.end - W.begin;
+    const int64_t nchunks = (total + 31) / 32;
+    const int64_t mychunks = nchunks > W.shard ? (nchunks - W.shard + W.nshards - 1) / W.nshards : 0;
+    const int64_t nloc = mychunks * 32;
+    const int64_t nthreads = (int64_t)gridDim.x * blockDim.x;
+    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
+    const int64_t tpos = (int64_t)lane * (nthreads >> 5) + warp;
+
+    int64_t kq = 0;                  // this lane's next root slot
+    bool have = false, done = false;
+    int u = 0, v = 0;
+    int64_t e = 0, pa = 0, ea = 0, pb = 0, eb = 0, su = 0, sv = 0;
+    int cnt = 0;                     // leaves in the warp buffer (warp-uniform)
+
+    auto flush = [&]() {
+        __syncwarp();
+        // (1) triple intersections + Venn, one leaf per lane (two passes if > 32)
+        for (int base = 0; base < cnt; base += 32) {
+            const int li = base + lane;
+            const bool mine = li < cnt;
+            int lu = 0, lv = 0, lw = 0, du = 0, dv = 0, dw = 0, t = 0;
+            int cuv = 0, cuw = 0, cvw = 0;
+            if (mine) {
+                lu = (int)s_leaf[wib][li][0]; lv = (int)s_leaf[wib][li][1]; lw = (int)s_leaf[wib][li][2];
+                cuv = __ldg(sup + s_leaf[wib][li][3]);
+                cuw = __ldg(sup + s_leaf[wib][li][4]);
+                cvw = __ldg(sup + s_leaf[wib][li][5]);
+                du = (int)(__ldg(G.offs + lu + 1) - __ldg(G.offs + lu));
+                dv = (int)(__ldg(G.offs + lv + 1) - __ldg(G.offs + lv));
+                dw = (int)(__ldg(G.offs + lw + 1) - __ldg(G.offs + lw));
+            }
+            const bool heavy = mine && du > kTriLight;
+            if (mine && !heavy) {
+                Cursor cv, cw;
+                cv.init(G, H, lv);
+                cw.init(G, H, lw);
+                const int64_t b0 = __ldg(G.offs + lu);
+                for (int i = 0; i < du; ++i) {
+                    const int x = __ldg(G.adj + b0 + i);
+                    if (cv.has(x) && cw.has(x)) ++t;
+                }
+            }
+            unsigned hb = __ballot_sync(FULLMASK, heavy);
+            while (hb) {
+                const int who = __ffs(hb) - 1;
+                hb &= hb - 1;
+                const int hu = __shfl_sync(FULLMASK, lu, who), hv = __shfl_sync(FULLMASK, lv, who);
+                const int hw = __shfl_sync(FULLMASK, lw, who), hd = __shfl_sync(FULLMASK, du, who);
+                const int64_t b0 = __ldg(G.offs + hu);
+                int tt = 0;
+                for (int s0 = 0; s0 < hd; s0 += 32) {
+                    bool hit = false;
+                    if (s0 + lane < hd) {
+                        const int x = __ldg(G.adj + b0 + s0 + lane);
+                        hit = member(G, H, hv, x) && member(G, H, hw, x);
+                    }
+                    tt += __popc(__ballot_sync(FULLMASK, hit));
+                }
+                if (lane == who) t = tt;
+            }
+            if (mine) {
+                int R[8];
+                R[7] = t;
+                R[3] = cuv - 1 - t;
+                R[5] = cuw - 1 - t;
+                R[6] = cvw - 1 - t;
+                R[1] = du - 2 - R[3] - R[5] - t;
+                R[2] = dv - 2 - R[3] - R[6] - t;
+                R[4] = dw - 2 - R[5] - R[6] - t;
+                uint32_t vq[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+#pragma unroll
+                for (int F = 1; F < 8; ++F)
+                    if (proj[F]) vq[proj[F]] += (uint32_t)R[F];
+                for (int k = 0; k < V; ++k) s_venn[wib][li][k] = vq[k];
+            }
+        }
+        __syncwarp();
+        // (2) fc over (leaf, program) pairs
+        const int pairs = cnt * nprog;
+        for (int tpair = lane; tpair < pairs; tpair += 32) {
+            const int li = tpair / nprog, pi = tpair - li * nprog;
+            uint32_t vloc[8];
+            for (int k = 0; k < V; ++k) vloc[k] = s_venn[wib][li][k];
+            const FringeProg fp = P.prog[pi];
+            bool o = false;
+            const u128 f = fc_dispatch<kTriStack>(vloc, q, fp, o);
+            acc.add(fp.pat, f, o);
+        }
+        nmatch += (lane == 0) ? (unsigned long long)cnt : 0ull;
+        cnt = 0;
+        __syncwarp();
+    };
+
+    for (;;) {
+        // refill: the next root of this lane that passes the degree filter
+        while (!have && !done) {
+            const int64_t L = kq * nthreads + tpos;
+            ++kq;
+            if (L >= nloc) { done = true; break; }
+            const int64_t tt = ((L >> 5) * W.nshards + W.shard) * 32 + (L & 31);
+            if (tt >= total) continue;
+            e = W.begin + tt;
+            u = __ldg(G.osrc + e);
+            v = __ldg(G.odst + e);
+            const int64_t ou = __ldg(G.offs + u), ou1 = __ldg(G.offs + u + 1);
+            const int64_t ov = __ldg(G.offs + v), ov1 = __ldg(G.offs + v + 1);
+            if (W.degfilter && ((int)(ou1 - ou) < P.mindeg[0] || (int)(ov1 - ov) < P.mindeg[1])) continue;
+            su = __ldg(O.split + u); pa = su; ea = ou1;
+            sv = __ldg(O.split + v); pb = sv; eb = ov1;
+            have = true;
+        }
+        if (__ballot_sync(FULLMASK, have) == 0) break;   // all lanes exhausted
+        // advance this lane's merge to its next triangle
+        bool found = false;
+        int w = 0;
+        int64_t fa = 0, fb = 0;
+        if (have) {
+            int x = pa < ea ? __ldg(G.adj + pa) : 0, y = pb < eb ? __ldg(G.adj + pb) : 0;
+            while (pa < ea && pb < eb) {
+                if (x < y) { if (++pa < ea) x = __ldg(G.adj + pa); }
+                else if (x > y) { if (++pb < eb) y = __ldg(G.adj + pb); }
+                else { found = true; w = x; fa = pa; fb = pb; ++pa; ++pb; break; }
+            }
+            if (!found) have = false;
+            if (found && W.degfilter) {
+                const int dw = (int)(__ldg(G.offs + w + 1) - __ldg(G.offs + w));
+                if (dw < P.mindeg[2]) found = false;
+            }
+        }
+        const unsigned fm = __ballot_sync(FULLMASK, found);
+        if (found) {
+            const int slot = cnt + __popc(fm & ((1u << lane) - 1));
+            s_leaf[wib][slot][0] = (uint32_t)u;
+            s_leaf[wib][slot][1] = (uint32_t)v;
+            s_leaf[wib][slot][2] = (uint32_t)w;
+            s_leaf[wib][slot][3] = (uint32_t)e;
+            s_leaf[wib][slot][4] = (uint32_t)(__ldg(O.oofs + u) + (fa - su));
+            s_leaf[wib][slot][5] = (uint32_t)(__ldg(O.oofs + v) + (fb - sv));
+        }
+        cnt += __popc(fm);
+        if (cnt >= 32) flush();
+    }
+    if (cnt) flush();
+    block_publish<NP>(acc, nmatch, S);
+}
+
+// ------------------------------------------------------------------------
 // Cores with p >= 2 vertices: one warp per root edge.
 template <int WARPS, int NP>
 __global__ void __launch_bounds__(WARPS * 32) core_kernel(GraphDev G, const CoreProg P, WorkDesc W,
@@ -806,13 +1039,15 @@ struct Kernels {
     static const void* vertex() { return (const void*)vertex_core_kernel<NP>; }
     static const void* edge() { return (const void*)edge_fc_kernel<NP>; }
     static const void* core() { return (const void*)core_kernel<kWarps, NP>; }
+    static const void* tri() { return (const void*)tri_core_kernel<NP>; }
 };
 
 // smallest NP in {1,2,4,8,16} holding npats
 int np_class(int npats) { return npats <= 1 ? 1 : npats <= 2 ? 2 : npats <= 4 ? 4 : npats <= 8 ? 8 : 16; }
 
 const void* kernel_for(int kind, int np) {
-#define FSGC_K(NPV) case NPV: return kind == 0 ? Kernels<NPV>::vertex() : kind == 1 ? Kernels<NPV>::edge() : Kernels<NPV>::core();
+#define FSGC_K(NPV) case NPV: return kind == 0 ? Kernels<NPV>::vertex() : kind == 1 ? Kernels<NPV>::edge() : \
+                                         kind == 2 ? Kernels<NPV>::core() : Kernels<NPV>::tri();
     switch (np) { FSGC_K(1) FSGC_K(2) FSGC_K(4) FSGC_K(8) FSGC_K(16) }
 #undef FSGC_K
     return nullptr;
@@ -989,6 +1224,12 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
         X.W = WorkDesc{b, e, opts.shard_index, opts.shard_count, 4,
                        (opts.flags & FSGC_FLAG_NO_DEGREE_FILTER) ? 0 : 1, nullptr};
         X.kind = cp.root_mode == ROOT_VERTEX ? 0 : (cp.p == 2 ? 1 : 2);
+        if (X.kind == 2 && cp.p == 3 && cp.back[2] == 3 && cp.root_mode == ROOT_ORIENTED && (cp.gt[2] & 2) &&
+            !tune("FSGC_NO_TRI", 0)) {
+            bool fits = true;   // Listing 5 stack bound of the triangle kernel
+            for (int k = 0; k < cp.nprog; ++k) fits = fits && cp.prog[k].depth <= kTriStack;
+            if (fits) X.kind = 3;
+        }
         if (X.kind == 0) {
             X.W.chunk = 256;
             int64_t work = (e - b + opts.shard_count - 1) / opts.shard_count;
@@ -1002,6 +1243,14 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
             X.grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy(kernel_for(1, X.npc), 256, 0),
                                                             (mine + 7) / 8));
             if (tune("FSGC_EDGE_BLOCKS", 0) > 0) X.grid = tune("FSGC_EDGE_BLOCKS", 0);
+            X.sup_bytes = (size_t)std::max<int64_t>(g->m, 1) * sizeof(int);
+        } else if (X.kind == 3) {
+            X.grid_sup = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy((const void*)support_kernel, 256, 0),
+                                                                (g->m + 255) / 256));
+            int64_t mine = ((e - b) + 31) / 32;
+            mine = (mine + opts.shard_count - 1) / opts.shard_count;
+            X.grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy(kernel_for(3, X.npc), kTriWarps * 32, 0),
+                                                            (mine + kTriWarps - 1) / kTriWarps));
             X.sup_bytes = (size_t)std::max<int64_t>(g->m, 1) * sizeof(int);
         } else {
             X.smem = (size_t)kWarps * 33 * (1u << cp.q) * sizeof(uint32_t);
@@ -1059,7 +1308,7 @@ extern "C" int fsgc_plan_enqueue(const fsgc_plan* P, void* workspace, void* raw_
         if (P->trace && X.kind == 1) W.trace = P->trace;
         const CoreProg& cp = X.plan.prog;
         FSGC_CUDA(cudaEventRecordWithFlags(P->ev[3 * pi], st, evflags));
-        if (X.kind == 1 && g->m > 0) {   // (A) per-edge common-neighbour counts (all edges)
+        if ((X.kind == 1 || X.kind == 3) && g->m > 0) {   // (A) per-edge common-neighbour counts
             support_kernel<<<(int)X.grid_sup, 256, 0, st>>>(G, O, g->m, dsup, dqueue2,
                                                              P->trace ? P->trace + (1 << 17) : nullptr);
             FSGC_CUDA(cudaGetLastError());
@@ -1070,10 +1319,14 @@ extern "C" int fsgc_plan_enqueue(const fsgc_plan* P, void* workspace, void* raw_
             void* args_v[] = {(void*)&G, (void*)&cp, (void*)&W, (void*)&S};
             void* args_e[] = {(void*)&G, (void*)&O, (void*)&cp, (void*)&W, (void*)&dsup, (void*)&S};
             void* args_c[] = {(void*)&G, (void*)&cp, (void*)&W, (void*)&S, (void*)&dqueue};
+            HubDev Hd{g->hub_base, g->hub_words, g->hub_bits};
+            void* args_t[] = {(void*)&G, (void*)&O, (void*)&Hd, (void*)&cp, (void*)&W, (void*)&dsup, (void*)&S};
             if (X.kind == 0)
                 FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(256), args_v, 0, st));
             else if (X.kind == 1)    // (B) fringe counts per root edge
                 FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(256), args_e, 0, st));
+            else if (X.kind == 3)
+                FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(kTriWarps * 32), args_t, 0, st));
             else
                 FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(kWarps * 32), args_c, X.smem, st));
         }
@@ -1096,7 +1349,7 @@ extern "C" int fsgc_plan_decode(const fsgc_plan* P, const void* raw, fsgc_result
         if (cudaEventElapsedTime(&ams, P->ev[3 * pi], P->ev[3 * pi + 1]) != cudaSuccess) ams = -1.f;
         if (cudaEventElapsedTime(&kms, P->ev[3 * pi + 1], P->ev[3 * pi + 2]) != cudaSuccess) kms = -1.f;
         cudaGetLastError();   // timing is best effort (e.g. events recorded inside a graph)
-        const int launches = (X.W.end > X.W.begin ? 1 : 0) + (X.kind == 1 && P->g->m > 0 ? 1 : 0);
+        const int launches = (X.W.end > X.W.begin ? 1 : 0) + ((X.kind == 1 || X.kind == 3) && P->g->m > 0 ? 1 : 0);
         for (size_t mi = 0; mi < X.plan.members.size(); ++mi) {
             fsgc_result& r = results[X.plan.members[mi]];
             r.raw.lo = acc[mi].lo;

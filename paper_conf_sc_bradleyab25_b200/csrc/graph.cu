@@ -15,6 +15,9 @@
 // osrc/odst int32[m] (SoA, sorted by (u, v)), order int32[n].
 #include <cub/cub.cuh>
 #include <atomic>
+#include <cstdlib>
+#include <vector>
+#include <algorithm>
 #include "devbuf.cuh"
 
 namespace {
@@ -113,6 +116,23 @@ __global__ void split_points(const int64_t* __restrict__ offs, const int32_t* __
         }
         split[v] = lo;
         out[v] = end - lo;
+    }
+}
+
+// bitmap rows of the hub vertices [hub_base, n)
+__global__ void hub_bitmaps(const int64_t* __restrict__ offs, const int32_t* __restrict__ adj, int64_t hub_base,
+                            int64_t n, int64_t words, uint32_t* __restrict__ bits) {
+    const int64_t beg = offs[hub_base], end = offs[n];
+    for (int64_t i = beg + blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < end;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        // row of entry i: binary search in offs over [hub_base, n)
+        int64_t lo = hub_base, hi = n;
+        while (hi - lo > 1) {
+            int64_t mid = (lo + hi) >> 1;
+            if (offs[mid] <= i) lo = mid; else hi = mid;
+        }
+        const int32_t x = adj[i];
+        atomicOr(bits + (lo - hub_base) * words + (x >> 5), 1u << (x & 31));
     }
 }
 
@@ -290,6 +310,39 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
     ka.release();
     kb.release();
     rank.release();
+
+    // hub bitmaps within a memory budget (default min(4 GiB, 5% of device
+    // memory); FSGC_HUB_BYTES overrides), only for degree >= kHubMinDeg
+    int64_t hub_base = n, hub_words = (n + 31) / 32;
+    DevBuf<uint32_t> hubs;
+    {
+        size_t free_b = 0, total_b = 0;
+        FSGC_CUDA(cudaMemGetInfo(&free_b, &total_b));
+        int64_t budget = std::min<int64_t>(4ll << 30, (int64_t)(total_b / 20));
+        if (const char* v = getenv("FSGC_HUB_BYTES")) budget = atoll(v);
+        budget = std::min<int64_t>(budget, (int64_t)(free_b / 4));
+        const int64_t per = hub_words * 4;
+        int64_t max_hubs = per > 0 ? budget / per : 0;
+        if (max_hubs > n) max_hubs = n;
+        if (max_hubs > 0 && M > 0) {
+            // smallest candidate base: the max_hubs highest ids; raise it until deg >= threshold
+            int64_t lo = n - max_hubs, hi = n;   // find first v in [lo, n) with deg(v) >= kHubMinDeg
+            const int64_t kHubMinDeg = 256;
+            while (lo < hi) {
+                int64_t mid = (lo + hi) / 2;
+                int64_t o2[2];
+                FSGC_CUDA(cudaMemcpy(o2, offs.ptr + mid, 2 * sizeof(int64_t), cudaMemcpyDeviceToHost));
+                if (o2[1] - o2[0] >= kHubMinDeg) hi = mid; else lo = mid + 1;
+            }
+            hub_base = lo;
+        }
+        if (hub_base < n) {
+            FSGC_CUDA(hubs.alloc((size_t)(n - hub_base) * hub_words, st));
+            FSGC_CUDA(cudaMemsetAsync(hubs.ptr, 0, (size_t)(n - hub_base) * hub_words * 4, st));
+            hub_bitmaps<<<grid_for(M), 256, 0, st>>>(offs.ptr, adj.ptr, hub_base, n, hub_words, hubs.ptr);
+            FSGC_CUDA(cudaGetLastError());
+        }
+    }
     int64_t maxdeg = 0;
     if (n > 0) {
         int64_t lastoffs[2] = {0, 0};
@@ -313,6 +366,9 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
     g->order = order.take();
     g->split = split.take();
     g->oofs = oofs.take();
+    g->hub_base = hub_base;
+    g->hub_words = hub_words;
+    g->hub_bits = hubs.take();
     g->device = dev;
     *out = g;
     return FSGC_OK;
@@ -350,5 +406,6 @@ extern "C" void fsgc_free_graph(fsgc_graph* g) {
     cudaFree(g->order);
     cudaFree(g->split);
     cudaFree(g->oofs);
+    cudaFree(g->hub_bits);
     delete g;
 }

@@ -29,6 +29,11 @@ struct fsgc_graph {
     int64_t* oofs = nullptr;     // [n+1] oriented offsets: oriented index of
                                  //       CSR position p >= split[u] is
                                  //       oofs[u] + p - split[u]
+    // hub bitmaps: vertices v >= hub_base (the highest-degree ones, ids are
+    // degree ordered) have a dense n-bit adjacency bitmap (O(1) membership)
+    int64_t hub_base = 0;        // == n when there are no hubs
+    int64_t hub_words = 0;       // 32-bit words per bitmap
+    uint32_t* hub_bits = nullptr;
     int device = 0;
 };
 
