@@ -20,10 +20,16 @@ from inputs.patterns import CONFIG_PATTERNS, PATTERNS  # noqa: E402
 def main():
     wl = sys.argv[1]
     names = sys.argv[2:] or CONFIG_PATTERNS[wl]
+    if os.environ.get("ROOTS"):        # count only a prefix of the root items
+        pass
     dev = torch.device("cuda", 0)
     t = time.time()
     if wl.startswith("rmat"):
         n, e = workload_edges(wl, device=dev)
+    elif wl.startswith("pl:"):          # pl:n:m:gamma:dmax
+        from inputs.graphs import powerlaw_edges
+        _, n_, m_, g_, d_ = wl.split(":")
+        n, e = int(n_), powerlaw_edges(int(n_), int(m_), float(g_), float(d_), seed=3)
     else:
         n, e = workload_edges(wl)
     torch.cuda.synchronize()
