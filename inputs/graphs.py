@@ -11,7 +11,9 @@ Workload shapes follow BASELINE.json ``configs`` and PAPER.md Table 1 (Sec. 5):
                   shaped like Table 1's "internet" row (configs[1])
   * ``rmat22``    RMAT scale 22, edge factor 16 (configs[2]; Table 1 lists
                   rmat16.sym and kron_g500-logn20 as the RMAT/Kronecker inputs)
-  * ``pl10m``     power-law, ~10M edges, d_max ~20k (configs[3]; in-2004-like)
+  * ``pl10m``     power-law, ~10M edges, d_max ~2.5k (configs[3]; d_max chosen so
+                  the Fig. 4 count stays below 2^128 -- DESIGN.md R11)
+  * ``rmat16``    RMAT scale 16, edge factor 8 (Table 1's rmat16.sym scale)
   * ``rmat26``    RMAT scale 26, edge factor 16, ~1B edges (configs[4])
 """
 import os
@@ -168,7 +170,7 @@ WORKLOADS = {
     "fig2": ("fig2", {}),
     "pl2k": ("powerlaw", dict(n=2000, m=10000, exponent=2.5, dmax=120, seed=1)),
     "internet": ("powerlaw", dict(n=124651, m=193620, exponent=2.1, dmax=151, seed=2)),
-    "pl10m": ("powerlaw", dict(n=1 << 20, m=10_000_000, exponent=2.2, dmax=20000, seed=3)),
+    "pl10m": ("powerlaw", dict(n=1 << 20, m=10_000_000, exponent=2.2, dmax=2500, seed=3)),
     "rmat16": ("rmat", dict(scale=16, edge_factor=8, seed=4)),
     "rmat22": ("rmat", dict(scale=22, edge_factor=16, seed=5)),
     "rmat26": ("rmat", dict(scale=26, edge_factor=16, seed=6)),
