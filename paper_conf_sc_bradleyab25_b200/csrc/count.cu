@@ -824,91 +824,266 @@ __global__ void __launch_bounds__(kTriWarps * 32) tri_core_kernel(GraphDev G, Or
 }
 
 // ------------------------------------------------------------------------
-// Cores with p >= 2 vertices: one warp per root edge.
-template <int WARPS, int NP>
-__global__ void __launch_bounds__(WARPS * 32) core_kernel(GraphDev G, const CoreProg P, WorkDesc W,
-                                                          const Sink S, unsigned long long* queue) {
+// General cores (p >= 3): one warp per root edge (atomic chunk queue, heavy
+// roots first), depth-first core matching with the Listing 7 ballot scheme.
+// Core matches are buffered per warp (32 leaves) and their Venn diagrams
+// computed ONE LANE PER LEAF (warp-cooperatively only for long lists):
+//   * anchors sorted by degree at run time; the lists of all but the two
+//     largest-degree anchors are scanned, each element tested against the
+//     later anchors (galloping cursors / hub bitmaps) -> raw histogram H
+//     (Sec. 3.6: only later anchors are searched, then corrected);
+//   * the last two anchors' pair count is the per-edge support when they are
+//     a core edge (else one more scan), singletons are degrees;
+//   * raw regions (core vertices included) follow by the Sec. 3.6 correction
+//     and inclusion-exclusion; each core vertex is then removed from the
+//     region of anchors it is adjacent to (e(x) excludes the core).
+// fc per (leaf, program) pair across the lanes: the partition-lattice terms
+// when every fringe type has k = 1, else Listing 5.
+struct TermDev {
+    const PartTerm* __restrict__ terms;
+    const int32_t* __restrict__ off;     // per program
+    const int32_t* __restrict__ cnt;     // per program, < 0: Listing 5
+};
+
+constexpr int kCoreWarps = 4;
+constexpr int kCoreLight = 48;   // scan work above this per leaf: warp-cooperative
+
+// oriented index of the graph edge {a, b} (must exist)
+__device__ __forceinline__ int64_t edge_index(const GraphDev& G, const OrientDev& O, int a, int b) {
+    const int lo = min(a, b), hi = max(a, b);
+    int64_t l = __ldg(O.split + lo), h = __ldg(G.offs + lo + 1);
+    while (l < h) {
+        const int64_t mid = (l + h) >> 1;
+        if (__ldg(G.adj + mid) < hi) l = mid + 1; else h = mid;
+    }
+    return __ldg(O.oofs + lo) + (l - __ldg(O.split + lo));
+}
+
+// partition-lattice fc: Z[A] = sum_{e >= A} venn[e]; fc = sum coef prod Z[mask]
+__device__ __noinline__ u128 fc_partition(const uint32_t* venn, int q, const PartTerm* __restrict__ T, int nt,
+                                          bool& ovf) {
+    int64_t Z[64];
+    const int V = 1 << q;
+    for (int A = 0; A < V; ++A) Z[A] = A ? venn[A] : 0;
+    for (int bb = 0; bb < q; ++bb)
+        for (int A = 0; A < V; ++A)
+            if (!(A >> bb & 1)) Z[A] += Z[A | (1 << bb)];
+    // 64-bit when the rising-factorial bound (N + s)^s < 2^62 holds, else 128
+    uint64_t N = (uint64_t)Z[0];
+    int smax = 0;
+    for (int i = 0; i < nt; ++i) {
+        int s = 0;
+        // number of types = sum of block sizes is constant; use nb of the finest term
+        s = T[i].nb;
+        smax = max(smax, s);
+    }
+    if ((int64_t)bitlen64(N + (uint64_t)smax) * smax <= 62) {
+        int64_t tot = 0;
+        for (int i = 0; i < nt; ++i) {
+            int64_t pr = T[i].coef;
+            for (int bb = 0; bb < T[i].nb; ++bb) pr *= Z[T[i].mask[bb]];
+            tot += pr;
+        }
+        return (u128)(uint64_t)tot;       // the count is non-negative
+    }
+    // signed 128-bit (two's complement); flag when the bound fails
+    if ((int64_t)bitlen64(N + (uint64_t)smax) * smax > 126) ovf = true;
+    u128 tot = 0;
+    for (int i = 0; i < nt; ++i) {
+        const bool neg = T[i].coef < 0;
+        u128 pr = (u128)(uint64_t)(neg ? -(int64_t)T[i].coef : T[i].coef);
+        for (int bb = 0; bb < T[i].nb; ++bb) pr *= (u128)(uint64_t)Z[T[i].mask[bb]];
+        tot = neg ? tot - pr : tot + pr;
+    }
+    return tot;
+}
+
+template <int NP>
+__global__ void __launch_bounds__(kCoreWarps * 32) core_kernel(GraphDev G, OrientDev O, HubDev H,
+                                                                const CoreProg P, WorkDesc W,
+                                                                const int* __restrict__ sup, TermDev TD,
+                                                                const Sink S, unsigned long long* queue) {
     extern __shared__ uint32_t smem[];
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-    const int q = P.q, V = 1 << q, p = P.p;
-    uint32_t* hist = smem + wib * (V * 33);
-    uint32_t* vbuf = hist + V;
-    int nbuf = 0;
+    const int q = P.q, V = 1 << q, p = P.p, nprog = P.nprog;
+    uint32_t* s_leaf = smem + wib * (32 * FSGC_MAXC);                       // [32][MAXC]
+    uint32_t* s_venn = smem + kCoreWarps * 32 * FSGC_MAXC + wib * (32 * V);  // [32][V]
     AccN<NP> acc;
     acc.init();
     unsigned long long nmatch = 0;
+    int cnt = 0;
 
     int emb[FSGC_MAXC];
     int64_t eoff[FSGC_MAXC];
     int edeg[FSGC_MAXC];
     int64_t cur[FSGC_MAXC], endp[FSGC_MAXC];
-    int pivl[FSGC_MAXC];
     uint32_t pend[FSGC_MAXC];
+    int pivl[FSGC_MAXC];
+    // core adjacency of positions (pattern core edges => graph edges)
+    uint32_t cadj[FSGC_MAXC];
+#pragma unroll
+    for (int i = 0; i < FSGC_MAXC; ++i) cadj[i] = 0;
+    for (int i = 1; i < p; ++i)
+        for (int j = 0; j < i; ++j)
+            if ((P.back[i] >> j) & 1) { cadj[i] |= 1u << j; cadj[j] |= 1u << i; }
 
-    // ---- fc over the buffered Venn diagrams, lanes over (diagram, program)
+    // ---- Venn of leaf li (one lane) -> s_venn
+    auto venn_lane = [&](int li, bool heavy_path) {
+        int a[FSGC_MAXQ], d[FSGC_MAXQ], pos[FSGC_MAXQ];
+        for (int bb = 0; bb < q; ++bb) {
+            pos[bb] = P.anchor_pos[bb];
+            a[bb] = (int)s_leaf[li * FSGC_MAXC + pos[bb]];
+            d[bb] = (int)(__ldg(G.offs + a[bb] + 1) - __ldg(G.offs + a[bb]));
+        }
+        int pi_[FSGC_MAXQ];                       // anchors by degree ascending
+        for (int bb = 0; bb < q; ++bb) pi_[bb] = bb;
+        for (int i = 1; i < q; ++i)
+            for (int j = i; j > 0 && d[pi_[j]] < d[pi_[j - 1]]; --j) { int t = pi_[j]; pi_[j] = pi_[j - 1]; pi_[j - 1] = t; }
+        int32_t R[64];
+        for (int k = 0; k < V; ++k) R[k] = 0;
+        const bool pair_adj = q >= 2 && ((cadj[pos[pi_[q - 2]]] >> pos[pi_[q - 1]]) & 1);
+        const int nscan = q >= 2 ? (pair_adj ? q - 2 : q - 1) : 0;
+        if (!heavy_path) {
+            for (int i = 0; i < nscan; ++i) {      // H[(1<<i) | later-mask], permuted bits
+                Cursor cs[FSGC_MAXQ];
+                for (int j = i + 1; j < q; ++j) cs[j].init(G, H, a[pi_[j]]);
+                const int64_t b0 = __ldg(G.offs + a[pi_[i]]);
+                for (int k = 0; k < d[pi_[i]]; ++k) {
+                    const int x = __ldg(G.adj + b0 + k);
+                    int m = 1 << i;
+                    for (int j = i + 1; j < q; ++j)
+                        if (cs[j].has(x)) m |= 1 << j;
+                    R[m] += 1;
+                }
+            }
+        } else {
+            for (int k = 0; k < V; ++k) R[k] = (int32_t)s_venn[li * V + k];   // H from the warp pass
+        }
+        // Sec. 3.6 correction: entries with lowest bit i < nscan are exact
+        // once the entries with a lower lowest bit are
+        for (int i = 0; i < nscan; ++i)
+            for (int t = V - 1; t > 0; --t) {
+                if ((__ffs(t) - 1) != i) continue;
+                const int low = (1 << i) - 1;
+                for (int E = low; E > 0; E = (E - 1) & low) R[t] -= R[E | t];
+            }
+        // the unscanned anchors: pair from the support, singletons from degrees
+        if (q >= 2 && pair_adj) {
+            const int i = q - 2, hb = (1 << (q - 2)) | (1 << (q - 1));
+            int r = __ldg(sup + edge_index(G, O, a[pi_[q - 2]], a[pi_[q - 1]]));
+            const int low = (1 << i) - 1;
+            for (int E = low; E > 0; E = (E - 1) & low) r -= R[E | hb];
+            R[hb] = r;
+        }
+        for (int i = nscan; i < q; ++i) {
+            int r = d[pi_[i]];
+            for (int t = V - 1; t > 0; --t)
+                if (((t >> i) & 1) && t != (1 << i)) r -= R[t];
+            R[1 << i] = r;
+        }
+        // remove the core vertices from their regions (e(x) excludes the core)
+        for (int y = 0; y < p; ++y) {
+            const int vy = (int)s_leaf[li * FSGC_MAXC + y];
+            int m = 0;
+            for (int i = 0; i < q; ++i) {
+                const int py = pos[pi_[i]];
+                if (py == y) continue;                        // no self loops
+                const bool adj = ((cadj[y] >> py) & 1) || member(G, H, a[pi_[i]], vy);
+                if (adj) m |= 1 << i;
+            }
+            if (m) R[m] -= 1;
+        }
+        // back to the programs' Venn bit order
+        for (int t = 1; t < V; ++t) {
+            int tb = 0;
+            for (int i = 0; i < q; ++i)
+                if ((t >> i) & 1) tb |= 1 << pi_[i];
+            s_venn[li * V + tb] = (uint32_t)R[t];
+        }
+        s_venn[li * V] = 0;
+    };
+
     auto flush = [&]() {
         __syncwarp();
-        const int tot = nbuf * P.nprog;
-        for (int t = lane; t < tot; t += 32) {
-            const int vi = t / P.nprog, pi = t - vi * P.nprog;
-            uint32_t vloc[1 << FSGC_MAXQ];
-            for (int e = 0; e < V; ++e) vloc[e] = vbuf[vi * V + e];
-            const FringeProg fp = P.prog[pi];
-            bool o = false;
-            u128 c = fc_dispatch<FSGC_FC_STACK>(vloc, q, fp, o);
-            acc.add(fp.pat, c, o);
+        const int li = lane;
+        bool mine = li < cnt, heavy = false;
+        if (mine) {                              // scan work of this leaf
+            int d2[FSGC_MAXQ], ds = 0;
+            for (int bb = 0; bb < q; ++bb) {
+                const int v = (int)s_leaf[li * FSGC_MAXC + P.anchor_pos[bb]];
+                d2[bb] = (int)(__ldg(G.offs + v + 1) - __ldg(G.offs + v));
+            }
+            for (int i = 1; i < q; ++i)
+                for (int j = i; j > 0 && d2[j] < d2[j - 1]; --j) { int t = d2[j]; d2[j] = d2[j - 1]; d2[j - 1] = t; }
+            for (int i = 0; i + 2 < q; ++i) ds += d2[i] * (q - 1 - i);
+            heavy = ds > kCoreLight * 2;
         }
-        nbuf = 0;
+        if (mine && !heavy) venn_lane(li, false);
+        unsigned hb = __ballot_sync(FULLMASK, heavy);
+        while (hb) {                             // warp-cooperative raw histogram
+            const int who = __ffs(hb) - 1;
+            hb &= hb - 1;
+            int a[FSGC_MAXQ], d[FSGC_MAXQ], pi_[FSGC_MAXQ];
+            for (int bb = 0; bb < q; ++bb) {
+                a[bb] = (int)s_leaf[who * FSGC_MAXC + P.anchor_pos[bb]];
+                d[bb] = (int)(__ldg(G.offs + a[bb] + 1) - __ldg(G.offs + a[bb]));
+                pi_[bb] = bb;
+            }
+            for (int i = 1; i < q; ++i)
+                for (int j = i; j > 0 && d[pi_[j]] < d[pi_[j - 1]]; --j) { int t = pi_[j]; pi_[j] = pi_[j - 1]; pi_[j - 1] = t; }
+            const bool pair_adj = q >= 2 && ((cadj[P.anchor_pos[pi_[q - 2]]] >> P.anchor_pos[pi_[q - 1]]) & 1);
+            const int nscan = q >= 2 ? (pair_adj ? q - 2 : q - 1) : 0;
+            for (int k = lane; k < V; k += 32) s_venn[who * V + k] = 0;
+            __syncwarp();
+            for (int i = 0; i < nscan; ++i) {
+                const int64_t b0 = __ldg(G.offs + a[pi_[i]]);
+                for (int s0 = 0; s0 < d[pi_[i]]; s0 += 32) {
+                    const bool valid = s0 + lane < d[pi_[i]];
+                    int m = 1 << i;
+                    if (valid) {
+                        const int x = __ldg(G.adj + b0 + s0 + lane);
+                        for (int j = i + 1; j < q; ++j)
+                            if (member(G, H, a[pi_[j]], x)) m |= 1 << j;
+                    }
+                    const unsigned act = __ballot_sync(FULLMASK, valid);
+                    if (valid) {
+                        const unsigned peers = __match_any_sync(act, m);
+                        if (lane == __ffs(peers) - 1) s_venn[who * V + m] += __popc(peers);
+                    }
+                    __syncwarp();
+                }
+            }
+            __syncwarp();
+            if (lane == who) venn_lane(who, true);
+            __syncwarp();
+        }
+        __syncwarp();
+        const int pairs = cnt * nprog;            // fc over (leaf, program) pairs
+        for (int tp = lane; tp < pairs; tp += 32) {
+            const int l2 = tp / nprog, pi = tp - l2 * nprog;
+            uint32_t vloc[1 << FSGC_MAXQ];
+            for (int k = 0; k < V; ++k) vloc[k] = s_venn[l2 * V + k];
+            bool o = false;
+            u128 f;
+            const int nt = __ldg(TD.cnt + pi);
+            if (nt >= 0) f = fc_partition(vloc, q, TD.terms + __ldg(TD.off + pi), nt, o);
+            else {
+                const FringeProg fp = P.prog[pi];
+                f = fc_dispatch<FSGC_FC_STACK>(vloc, q, fp, o);
+            }
+            acc.add(P.prog[pi].pat, f, o);
+        }
+        if (lane == 0) nmatch += cnt;
+        cnt = 0;
         __syncwarp();
     };
 
-    // ---- Venn diagram of the current core match into vbuf[nbuf]
     auto leaf = [&]() {
-        if (lane == 0) ++nmatch;
-        uint32_t* R = vbuf + nbuf * V;
-        for (int t = lane; t < V; t += 32) hist[t] = 0;
-        __syncwarp();
-        for (int i = 0; i < q; ++i) {
-            const int pi = P.anchor_pos[i];
-            const int32_t* __restrict__ Li = G.adj + eoff[pi];
-            const int li = edeg[pi];
-            for (int b0 = 0; b0 < li; b0 += 32) {
-                const int ix = b0 + lane;
-                bool valid = ix < li;
-                const int x = valid ? __ldg(Li + ix) : -1;
 #pragma unroll
-                for (int j = 0; j < FSGC_MAXC; ++j)
-                    if (j < p && x == emb[j]) valid = false;   // e(x) excludes the core
-                uint32_t m = 1u << i;
-                if (valid)
-                    for (int j = i + 1; j < q; ++j) {
-                        const int pj = P.anchor_pos[j];
-                        if (contains(G.adj + eoff[pj], edeg[pj], x)) m |= 1u << j;
-                    }
-                const unsigned act = __ballot_sync(FULLMASK, valid);
-                if (valid) {
-                    const unsigned peers = __match_any_sync(act, m);
-                    if (lane == __ffs(peers) - 1) hist[m] += __popc(peers);
-                }
-                __syncwarp();
-            }
-        }
-        // regions: entries whose lowest bit is i are exact once the regions
-        // with a lower lowest bit are known (Sec. 3.6 "we computationally
-        // correct them")
-        for (int i = 0; i < q; ++i) {
-            for (int t = lane; t < V; t += 32) {
-                if (t == 0 || (__ffs(t) - 1) != i) continue;
-                int r = (int)hist[t];
-                const int low = (1 << i) - 1;
-                for (int E = low; E > 0; E = (E - 1) & low) r -= (int)R[E | t];
-                R[t] = (uint32_t)r;
-            }
-            __syncwarp();
-        }
-        if (lane == 0) R[0] = 0;
-        __syncwarp();
-        if (++nbuf == 32) flush();
+        for (int j = 0; j < FSGC_MAXC; ++j)
+            if (lane == j && j < p) s_leaf[cnt * FSGC_MAXC + j] = (uint32_t)emb[j];
+        ++cnt;
+        if (cnt == 32) flush();
     };
 
     auto init_level = [&](int l) {
@@ -947,7 +1122,6 @@ __global__ void __launch_bounds__(WARPS * 32) core_kernel(GraphDev G, const Core
             emb[0] = u0; eoff[0] = G.offs[u0]; edeg[0] = (int)(G.offs[u0 + 1] - eoff[0]);
             emb[1] = u1; eoff[1] = G.offs[u1]; edeg[1] = (int)(G.offs[u1 + 1] - eoff[1]);
             if (W.degfilter && (edeg[0] < P.mindeg[0] || edeg[1] < P.mindeg[1])) continue;
-            if (p == 2) { leaf(); continue; }
             int lvl = 2;
             init_level(2);
             while (lvl >= 2) {
@@ -965,8 +1139,7 @@ __global__ void __launch_bounds__(WARPS * 32) core_kernel(GraphDev G, const Core
                     if (ok) {
                         const int piv = pivl[lvl];
                         for (int j = 0; j < lvl && ok; ++j)
-                            if ((P.back[lvl] >> j & 1) && j != piv)
-                                ok = contains(G.adj + eoff[j], edeg[j], x);
+                            if ((P.back[lvl] >> j & 1) && j != piv) ok = member(G, H, emb[j], x);
                     }
                     pend[lvl] = __ballot_sync(FULLMASK, ok);
                     cur[lvl] += 32;   // candidates are re-read from adj[cur - 32 + who]
@@ -987,7 +1160,7 @@ __global__ void __launch_bounds__(WARPS * 32) core_kernel(GraphDev G, const Core
             }
         }
     }
-    if (nbuf) flush();
+    if (cnt) flush();
     block_publish<NP>(acc, nmatch, S);
 }
 
@@ -1038,7 +1211,7 @@ template <int NP>
 struct Kernels {
     static const void* vertex() { return (const void*)vertex_core_kernel<NP>; }
     static const void* edge() { return (const void*)edge_fc_kernel<NP>; }
-    static const void* core() { return (const void*)core_kernel<kWarps, NP>; }
+    static const void* core() { return (const void*)core_kernel<NP>; }
     static const void* tri() { return (const void*)tri_core_kernel<NP>; }
 };
 
@@ -1165,6 +1338,7 @@ struct PassExec {
     size_t smem = 0;
     WorkDesc W{};
     size_t ws_off = 0, sup_bytes = 0, parts_off = 0, bytes = 0;
+    int term_base = 0;         // index of this pass's programs in the term offset/count arrays
     bool whole = true;
 };
 }  // namespace
@@ -1178,9 +1352,15 @@ struct fsgc_plan {
     int device = 0;
     std::vector<cudaEvent_t> ev;   // 3 per pass
     unsigned long long* trace = nullptr;
+    PartTerm* terms_dev = nullptr;   // partition-lattice terms of all programs
+    int32_t* off_dev = nullptr;
+    int32_t* cnt_dev = nullptr;
     ~fsgc_plan() {
         for (auto e : ev) cudaEventDestroy(e);
         if (trace) cudaFree(trace);
+        if (terms_dev) cudaFree(terms_dev);
+        if (off_dev) cudaFree(off_dev);
+        if (cnt_dev) cudaFree(cnt_dev);
     }
 };
 
@@ -1253,11 +1433,12 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
                                                             (mine + kTriWarps - 1) / kTriWarps));
             X.sup_bytes = (size_t)std::max<int64_t>(g->m, 1) * sizeof(int);
         } else {
-            X.smem = (size_t)kWarps * 33 * (1u << cp.q) * sizeof(uint32_t);
+            X.smem = (size_t)kCoreWarps * (32 * FSGC_MAXC + 32 * (1u << cp.q)) * sizeof(uint32_t);
             int64_t nchunks = ((e - b) + X.W.chunk - 1) / X.W.chunk;
             int64_t mine = (nchunks + opts.shard_count - 1) / opts.shard_count;
-            X.grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy(kernel_for(2, X.npc), kWarps * 32, X.smem),
-                                                            (mine + kWarps - 1) / kWarps));
+            X.grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy(kernel_for(2, X.npc), kCoreWarps * 32, X.smem),
+                                                            (mine + kCoreWarps - 1) / kCoreWarps));
+            X.sup_bytes = (size_t)std::max<int64_t>(g->m, 1) * sizeof(int);
         }
         X.parts_off = (kHdrBytes + X.sup_bytes + 255) & ~(size_t)255;
         X.bytes = (X.parts_off + (size_t)X.grid * sizeof(BlockPartial) + 255) & ~(size_t)255;
@@ -1266,6 +1447,27 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
         P->passes.push_back(X);
     }
     P->ws_bytes = off;
+    {   // partition-lattice term tables -> device
+        std::vector<PartTerm> all;
+        std::vector<int32_t> offs, cnts;
+        for (auto& X : P->passes) {
+            X.term_base = (int)offs.size();
+            for (int k = 0; k < X.plan.prog.nprog; ++k) {
+                const auto& T = X.plan.terms[k];
+                offs.push_back((int32_t)all.size());
+                cnts.push_back(T.empty() ? -1 : (int32_t)T.size());
+                all.insert(all.end(), T.begin(), T.end());
+            }
+        }
+        if (all.empty()) all.push_back(PartTerm{});
+        if (offs.empty()) { offs.push_back(0); cnts.push_back(-1); }
+        FSGC_CUDA(cudaMalloc(&P->terms_dev, all.size() * sizeof(PartTerm)));
+        FSGC_CUDA(cudaMalloc(&P->off_dev, offs.size() * sizeof(int32_t)));
+        FSGC_CUDA(cudaMalloc(&P->cnt_dev, cnts.size() * sizeof(int32_t)));
+        FSGC_CUDA(cudaMemcpy(P->terms_dev, all.data(), all.size() * sizeof(PartTerm), cudaMemcpyHostToDevice));
+        FSGC_CUDA(cudaMemcpy(P->off_dev, offs.data(), offs.size() * sizeof(int32_t), cudaMemcpyHostToDevice));
+        FSGC_CUDA(cudaMemcpy(P->cnt_dev, cnts.data(), cnts.size() * sizeof(int32_t), cudaMemcpyHostToDevice));
+    }
     P->ev.resize(3 * P->passes.size());
     for (auto& ev : P->ev) FSGC_CUDA(cudaEventCreate(&ev));
     if (tune("FSGC_TRACE", 0)) {
@@ -1308,7 +1510,7 @@ extern "C" int fsgc_plan_enqueue(const fsgc_plan* P, void* workspace, void* raw_
         if (P->trace && X.kind == 1) W.trace = P->trace;
         const CoreProg& cp = X.plan.prog;
         FSGC_CUDA(cudaEventRecordWithFlags(P->ev[3 * pi], st, evflags));
-        if ((X.kind == 1 || X.kind == 3) && g->m > 0) {   // (A) per-edge common-neighbour counts
+        if (X.kind != 0 && g->m > 0) {   // (A) per-edge common-neighbour counts
             support_kernel<<<(int)X.grid_sup, 256, 0, st>>>(G, O, g->m, dsup, dqueue2,
                                                              P->trace ? P->trace + (1 << 17) : nullptr);
             FSGC_CUDA(cudaGetLastError());
@@ -1318,8 +1520,10 @@ extern "C" int fsgc_plan_enqueue(const fsgc_plan* P, void* workspace, void* raw_
             const void* fn = kernel_for(X.kind, X.npc);
             void* args_v[] = {(void*)&G, (void*)&cp, (void*)&W, (void*)&S};
             void* args_e[] = {(void*)&G, (void*)&O, (void*)&cp, (void*)&W, (void*)&dsup, (void*)&S};
-            void* args_c[] = {(void*)&G, (void*)&cp, (void*)&W, (void*)&S, (void*)&dqueue};
             HubDev Hd{g->hub_base, g->hub_words, g->hub_bits};
+            TermDev TD{P->terms_dev, P->off_dev + X.term_base, P->cnt_dev + X.term_base};
+            void* args_c[] = {(void*)&G, (void*)&O, (void*)&Hd, (void*)&cp, (void*)&W, (void*)&dsup, (void*)&TD,
+                              (void*)&S, (void*)&dqueue};
             void* args_t[] = {(void*)&G, (void*)&O, (void*)&Hd, (void*)&cp, (void*)&W, (void*)&dsup, (void*)&S};
             if (X.kind == 0)
                 FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(256), args_v, 0, st));
@@ -1328,7 +1532,7 @@ extern "C" int fsgc_plan_enqueue(const fsgc_plan* P, void* workspace, void* raw_
             else if (X.kind == 3)
                 FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(kTriWarps * 32), args_t, 0, st));
             else
-                FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(kWarps * 32), args_c, X.smem, st));
+                FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(kCoreWarps * 32), args_c, X.smem, st));
         }
         FSGC_CUDA(cudaEventRecordWithFlags(P->ev[3 * pi + 2], st, evflags));
         FSGC_CUDA(cudaMemcpyAsync((unsigned char*)raw_out + pi * kRawPassBytes, base, kRawPassBytes - 8,
@@ -1349,7 +1553,7 @@ extern "C" int fsgc_plan_decode(const fsgc_plan* P, const void* raw, fsgc_result
         if (cudaEventElapsedTime(&ams, P->ev[3 * pi], P->ev[3 * pi + 1]) != cudaSuccess) ams = -1.f;
         if (cudaEventElapsedTime(&kms, P->ev[3 * pi + 1], P->ev[3 * pi + 2]) != cudaSuccess) kms = -1.f;
         cudaGetLastError();   // timing is best effort (e.g. events recorded inside a graph)
-        const int launches = (X.W.end > X.W.begin ? 1 : 0) + ((X.kind == 1 || X.kind == 3) && P->g->m > 0 ? 1 : 0);
+        const int launches = (X.W.end > X.W.begin ? 1 : 0) + (X.kind != 0 && P->g->m > 0 ? 1 : 0);
         for (size_t mi = 0; mi < X.plan.members.size(); ++mi) {
             fsgc_result& r = results[X.plan.members[mi]];
             r.raw.lo = acc[mi].lo;

@@ -89,8 +89,18 @@ struct CoreProg {
     uint8_t ek[FSGC_MAXPROG], el[FSGC_MAXPROG], em[FSGC_MAXPROG];
 };
 
+// fc of a program whose fringe types all have k = 1, by Moebius inversion on
+// the partition lattice of its s types: fc = sum_pi coef(pi) prod_B Z[mask_B],
+// Z[A] = sum of the Venn entries covering A; coef = prod (-1)^(|B|-1)(|B|-1)!
+struct PartTerm {
+    int32_t coef;
+    uint8_t nb;                 // blocks
+    uint8_t mask[7];            // Venn-bit anchor mask of each block
+};
+
 struct PassPlan {
     CoreProg prog;
+    std::vector<std::vector<PartTerm>> terms;   // per program (empty: Listing 5)
     std::vector<int> members;          // indices into the caller's pattern array
     std::vector<uint64_t> divisor;     // per member: count = raw / divisor
     int root_pattern_vertex[FSGC_MAXPATS];

@@ -454,6 +454,50 @@ int fsgc_build_pass(const fsgc_pattern* const* pats, const std::vector<int>& mem
         for (int i = 0; i < p; ++i) cp.mindeg[i] = std::min(cp.mindeg[i], att[i]);
     }
     for (int i = 0; i < p; ++i) cp.mindeg[i] += popc64(cadj[i]);
+    // partition-lattice term tables for programs with all k = 1 and <= 7 types
+    plan->terms.assign(cp.nprog, {});
+    for (int k = 0; k < cp.nprog; ++k) {
+        const FringeProg& fp = cp.prog[k];
+        bool ones = fp.s >= 1 && fp.s <= 7;
+        for (int t = 0; t < fp.s && ones; ++t) ones = fp.k[t] == 1;
+        if (!ones) continue;
+        const int sN = fp.s;
+        std::map<std::vector<uint8_t>, int64_t> acc;
+        int rgs[7] = {0};   // restricted growth string
+        for (;;) {
+            int nb = 0;
+            for (int i = 0; i < sN; ++i) nb = std::max(nb, rgs[i] + 1);
+            std::vector<uint8_t> masks(nb, 0);
+            std::vector<int> sz(nb, 0);
+            for (int i = 0; i < sN; ++i) { masks[rgs[i]] |= fp.anch[i]; sz[rgs[i]]++; }
+            int64_t coef = 1;
+            for (int b = 0; b < nb; ++b) {
+                int64_t f = 1;
+                for (int j = 2; j < sz[b]; ++j) f *= j;
+                coef *= ((sz[b] - 1) & 1) ? -f : f;
+            }
+            std::sort(masks.begin(), masks.end());
+            acc[masks] += coef;
+            // next restricted growth string
+            int i = sN - 1;
+            for (; i > 0; --i) {
+                int mx = 0;
+                for (int j = 0; j < i; ++j) mx = std::max(mx, rgs[j]);
+                if (rgs[i] <= mx) { ++rgs[i]; break; }
+                rgs[i] = 0;
+            }
+            if (i == 0) break;
+            for (int j = i + 1; j < sN; ++j) rgs[j] = 0;
+        }
+        for (auto& kv : acc) {
+            if (kv.second == 0) continue;
+            PartTerm tm{};
+            tm.coef = (int32_t)kv.second;
+            tm.nb = (uint8_t)kv.first.size();
+            for (size_t b = 0; b < kv.first.size(); ++b) tm.mask[b] = kv.first[b];
+            plan->terms[k].push_back(tm);
+        }
+    }
     if (p == 1) cp.root_mode = ROOT_VERTEX;
     else if (cp.gt[1] & 1) cp.root_mode = ROOT_ORIENTED;
     else cp.root_mode = ROOT_DIRECTED;

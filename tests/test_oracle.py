@@ -319,3 +319,41 @@ def test_core_matches():
     assert oracle.core_matches(g, P.n, P.edges) == int(A.sum()) // 2          # edge core
     P = PATTERNS["clique4"]
     assert oracle.core_matches(g, P.n, P.edges) == int(np.trace(np.linalg.matrix_power(A, 3))) // 6
+
+
+def _set_partitions(items):
+    if not items:
+        yield []
+        return
+    first, rest = items[0], items[1:]
+    for p in _set_partitions(rest):
+        yield [[first]] + p
+        for i in range(len(p)):
+            yield p[:i] + [[first] + p[i]] + p[i + 1:]
+
+
+def test_partition_lattice_identity_equals_listing5():
+    """The GPU evaluates fc for programs whose fringe types all have k = 1 by
+    Moebius inversion on the partition lattice: #(distinct x_t in U_t) =
+    sum_pi prod_B (-1)^(|B|-1) (|B|-1)! |cap_{t in B} U_t|.  Pin that identity
+    against Listing 5 (oracle.fc) on random Venn diagrams, q <= 4."""
+    from math import factorial
+    rng = random.Random(21)
+    for _ in range(250):
+        q = rng.randint(1, 4)
+        venn = [0] + [rng.randint(0, 4) for _ in range((1 << q) - 1)]
+        s = rng.randint(1, min(5, (1 << q) - 1))
+        anch = rng.sample(range(1, 1 << q), s)
+        Z = {}
+        for A in range(1 << q):
+            Z[A] = sum(venn[e] for e in range(1, 1 << q) if e & A == A)
+        tot = 0
+        for part in _set_partitions(list(range(s))):
+            term = 1
+            for B in part:
+                mask = 0
+                for t in B:
+                    mask |= anch[t]
+                term *= (-1) ** (len(B) - 1) * factorial(len(B) - 1) * Z[mask]
+            tot += term
+        assert tot == oracle.fc(list(venn), q, anch, [1] * s)
