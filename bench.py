@@ -317,22 +317,29 @@ def main():
             ev1[s].record(stream)
             torch.cuda.synchronize()
         assert [r.count for r in res] == counts
-        kms.append(res[0].kernel_ms)
-        ams.append(res[0].aux_ms)
-        launches += res[0].kernel_launches
+        passes = {}
+        for r in res:
+            passes[r.pass_index] = r
+        kms.append({k: r.kernel_ms for k, r in passes.items()})
+        ams.append({k: r.aux_ms for k, r in passes.items()})
+        launches += sum(r.kernel_launches for r in passes.values())
     step_ms = [a.elapsed_time(b) for a, b in zip(ev0, ev1)]
     clocks = sampler.stop()
     total_ms = sum(step_ms)
+    pass_ids = sorted(kms[0].keys())
+    kms_sum = {k: sum(x[k] for x in kms) for k in pass_ids}
+    ams_sum = {k: sum(x[k] for x in ams) for k in pass_ids}
     if world > 1:
-        t = torch.tensor([total_ms, sum(kms), sum(ams)], dtype=torch.float64, device=dev)
+        t = torch.tensor([total_ms] + [kms_sum[k] for k in pass_ids] + [ams_sum[k] for k in pass_ids],
+                         dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        total_ms, kms_sum, ams_sum = t.tolist()
-    else:
-        kms_sum, ams_sum = sum(kms), sum(ams)
+        vals = t.tolist()
+        total_ms = vals[0]
+        kms_sum = {k: vals[1 + i] for i, k in enumerate(pass_ids)}
+        ams_sum = {k: vals[1 + len(pass_ids) + i] for i, k in enumerate(pass_ids)}
     ms_per_step = total_ms / args.steps
     value = core_matches / (ms_per_step / 1e3)
-    kernel_ms = kms_sum / args.steps
-    aux_ms = ams_sum / args.steps
+    kind_of = {r.pass_index: r.pass_kind for r in res}
 
     # ---- roofline of the dominant kernel: algorithmic
     # bytes per launch / CUDA-event duration, against the measured HBM peak
@@ -349,9 +356,21 @@ def main():
     sup_bytes = 40.0 * m + 4.0 * float((out * out).sum() + (indeg * out).sum())
     # fc pass: per root edge 8 B (u,v) + 32 B (4 offsets) + 4 B support
     fc_bytes = 44.0 * m * share
-    kernels = [("edge_fc_kernel (Venn + Sec. 3.1 fc, lane per root edge)", fc_bytes, kernel_ms),
-               ("support_kernel (per-edge |N(u)&N(v)| by oriented listing)", sup_bytes, aux_ms)]
-    kernels.sort(key=lambda k: -k[2])
+    # general / triangle core passes: compulsory graph bytes (CSR + oriented
+    # view + supports read once) -- these kernels are latency/ALU bound
+    graph_bytes = (8.0 * 2 * m + 8.0 * (n + 1) + 8.0 * m + 4.0 * m + 16.0 * n) * share
+    names = {0: "vertex_core_kernel", 1: "edge_fc_kernel (Venn + Sec. 3.1 fc, lane per root edge)",
+             2: "core_kernel (general core: DFS + min-list Venn + fc)",
+             3: "tri_core_kernel (triangle core: listing + Venn + fc)"}
+    kernels = []
+    for k in pass_ids:
+        kind = kind_of[k]
+        byts = fc_bytes if kind == 1 else (8.0 * (n + 1) * share if kind == 0 else graph_bytes)
+        kernels.append((names[kind] + f" [pass {k}]", byts, kms_sum[k] / args.steps))
+        if kind != 0:
+            kernels.append((f"support_kernel (per-edge |N(u)&N(v)| by oriented listing) [pass {k}]",
+                            sup_bytes, ams_sum[k] / args.steps))
+    kernels.sort(key=lambda kk: -kk[2])
     peak, peak_src = measured_peaks()
     def roof(name, byts, ms):
         traffic = ncu_traffic(args.workload, name)

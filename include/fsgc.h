@@ -173,6 +173,9 @@ typedef struct {
     float aux_ms;           /* device time of the auxiliary per-edge support
                                pass (edge cores), 0 otherwise                 */
     int32_t kernel_launches;/* kernels launched for this pattern's pass       */
+    int32_t pass_index;     /* patterns with equal pass_index shared one pass */
+    int32_t pass_kind;      /* 0 vertex core, 1 edge core (support + fc),
+                               2 general core, 3 triangle core (support + tri) */
 } fsgc_result;
 
 typedef struct {

@@ -73,6 +73,7 @@ class Result(C.Structure):
         ("count", u128), ("raw", u128), ("divisor", C.c_uint64), ("core_matches", C.c_uint64),
         ("overflow", C.c_int32), ("root_pattern_vertex", C.c_int32),
         ("kernel_ms", C.c_float), ("aux_ms", C.c_float), ("kernel_launches", C.c_int32),
+        ("pass_index", C.c_int32), ("pass_kind", C.c_int32),
     ]
 
 

@@ -113,6 +113,8 @@ class CountResult:
     kernel_ms: float = 0.0
     aux_ms: float = 0.0
     kernel_launches: int = 0
+    pass_index: int = 0
+    pass_kind: int = 0
 
 
 def fsgc_load_graph(edges, num_vertices, stream=None) -> Graph:
@@ -189,7 +191,7 @@ def _results(res, whole):
             count=(r.count.value if (whole and not r.overflow) else None), raw=r.raw.value,
             divisor=r.divisor, core_matches=r.core_matches, overflow=bool(r.overflow),
             root_pattern_vertex=r.root_pattern_vertex, kernel_ms=r.kernel_ms, aux_ms=r.aux_ms,
-            kernel_launches=r.kernel_launches))
+            kernel_launches=r.kernel_launches, pass_index=r.pass_index, pass_kind=r.pass_kind))
     return out
 
 

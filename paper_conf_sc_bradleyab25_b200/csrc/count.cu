@@ -1565,6 +1565,8 @@ extern "C" int fsgc_plan_decode(const fsgc_plan* P, const void* raw, fsgc_result
             r.kernel_ms = kms;
             r.aux_ms = ams;
             r.kernel_launches = launches;
+            r.pass_index = (int32_t)pi;
+            r.pass_kind = X.kind;
             if (X.whole) {
                 int rc = fsgc_finalize(r.raw, r.divisor, r.overflow, &r.count, &r.overflow);
                 if (rc) return rc;
