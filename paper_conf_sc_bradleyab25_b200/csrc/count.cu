@@ -405,26 +405,32 @@ __device__ __forceinline__ int support_warp(const int32_t* __restrict__ adj, con
     return c;
 }
 
+// Roots are taken in the graph's support order (oriented edges sorted by
+// merge length out(u) + out(v), fsgc_graph.sorder): warp w takes the 32-root
+// chunks w, w + NW, ..., so the lanes of a warp run merges of similar length
+// (little divergence) and the heaviest chunks, at the end, spread over warps.
 __global__ void __launch_bounds__(256) support_kernel(GraphDev G, OrientDev O, int64_t m, int* __restrict__ sup,
-                                                      unsigned long long* queue, unsigned long long* trace) {
+                                                      const int32_t* __restrict__ sorder,
+                                                      const int32_t* __restrict__ ssrc,
+                                                      const int32_t* __restrict__ sdst,
+                                                      unsigned long long* trace) {
     const int lane = threadIdx.x & 31;
     const unsigned long long t_start = trace ? gtimer() : 0;
     int nch = 0;
-    const int64_t nthreads = (int64_t)gridDim.x * blockDim.x;
-    const int64_t NW = nthreads >> 5;
+    const int64_t NW = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t tpos = (int64_t)lane * NW + warp;   // transposed: hubs spread over warps
-    (void)queue;
-    for (int64_t t0 = 0; t0 < m; t0 += nthreads) {
+    const int64_t nchunks = (m + 31) >> 5;
+    for (int64_t ch = warp; ch < nchunks; ch += NW) {
         ++nch;
-        const int64_t t = t0 + tpos;
+        const int64_t t = ch * 32 + lane;
         const bool valid = t < m;
-        const int64_t e = valid ? t : 0;
+        int64_t e = 0;
         int u = 0, v = 0, nu = 0, nv = 0;
         int64_t su = 0, sv = 0;
         if (valid) {
-            u = __ldg(G.osrc + e);
-            v = __ldg(G.odst + e);
+            e = __ldg(sorder + t);
+            u = __ldg(ssrc + t);
+            v = __ldg(sdst + t);
             su = __ldg(O.split + u); nu = (int)(__ldg(G.offs + u + 1) - su);
             sv = __ldg(O.split + v); nv = (int)(__ldg(G.offs + v + 1) - sv);
         }
@@ -474,120 +480,193 @@ __device__ __forceinline__ int64_t edge_of_entry(const GraphDev& G, const Orient
 
 constexpr int kEdgeILP = 4;   // root edges per lane per iteration (independent loads in flight)
 
+// Sec. 3.1's closed form over binomial rows.  With the multinomial identity
+//   C(n,i) C(n-i,j) C(n-i-j,m) = C(n, i+j+m) (i+j+m)! / (i! j! m!)
+// the last displayed formula of Sec. 3.1 becomes
+//   fc(k,l,m) = sum_{i<=k, j<=l} C(nu,k-i) C(nv,l-j) C(nuv,i+j+m) (i+j+m)!/(i! j! m!),
+// a sum of products of three row entries Ra[a] = C(nu,a), Rb[b] = C(nv,b),
+// Rc[c] = C(nuv,c).  The host lists every (pattern, a, b, c, coefficient)
+// term of every program of the pass once (terms of one pattern merged), so a
+// root costs three short rows plus one multiply-add chain per term, shared by
+// all patterns and programs of the pass.
+constexpr int kMaxEdgeTerms = 160;
+constexpr int kMaxRowEntries = 24;   // (ka+1) + (kb+1) + (kc+1)
+struct EdgeTerm {
+    uint8_t a, b, c, pat;
+    uint32_t pad;
+    uint64_t coef;
+};
+struct EdgeTerms {
+    int32_t n;              // terms; 0: table path off (checked per-program path)
+    int32_t ka, kb, kc;     // row lengths - 1
+    int32_t kmax;           // max fringes of one program (64-bit bound, fc.cuh)
+    int32_t pad;
+    EdgeTerm t[kMaxEdgeTerms];
+};
+
+// exact division by t <= 63 of a multiple of t: shift out the 2-adic part,
+// multiply by the inverse of the odd part mod 2^64 (filled by ensure_binom_table)
+__constant__ uint64_t c_inv_odd[64];     // mod 2^64
+__constant__ uint64_t c_inv_odd_hi[64];  // high words of the inverses mod 2^128
+__constant__ uint32_t c_tz[64];
+
+__device__ __forceinline__ uint64_t inv_odd(int t, uint64_t) { return c_inv_odd[t]; }
+__device__ __forceinline__ u128 inv_odd(int t, u128) { return u128_make(c_inv_odd[t], c_inv_odd_hi[t]); }
+
+// R[t * stride] = C(n, t), t = 0..K, in arithmetic mod 2^bits(W); exact when
+// n^K < 2^(bits - 1) (caller's bound): every r * (n - t + 1) <= n^t then fits
+template <class W>
+__device__ __forceinline__ void binom_row(uint64_t n, int K, W* R, int stride) {
+    W r = 1;
+    R[0] = 1;
+    for (int t = 1; t <= K; ++t) {
+        r = ((r * (W)(n - (uint64_t)t + 1)) >> c_tz[t]) * inv_odd(t, r);
+        R[t * stride] = r;
+    }
+}
+
+// every term of the pass on one root's rows, arithmetic mod 2^bits(W): exact
+// because every program's fc is below N^K < 2^(bits - 1) (caller's bound) and
+// a pattern has at most |Aut(edge)| = 2 programs, so each pattern's sum fits
+template <class W, int NP>
+__device__ __forceinline__ void edge_terms_eval(uint64_t nu, uint64_t nv, uint64_t nuv, const EdgeTerms& T, W* R,
+                                                int stride, AccN<NP>& acc) {
+    W* Ra = R;
+    W* Rb = Ra + (T.ka + 1) * stride;
+    W* Rc = Rb + (T.kb + 1) * stride;
+    binom_row<W>(nu, T.ka, Ra, stride);
+    binom_row<W>(nv, T.kb, Rb, stride);
+    binom_row<W>(nuv, T.kc, Rc, stride);
+    W sum = 0;
+    int cur = T.t[0].pat;
+    for (int t = 0; t < T.n; ++t) {
+        const EdgeTerm e = T.t[t];
+        if (e.pat != cur) { acc.add(cur, (u128)sum, false); sum = 0; cur = e.pat; }
+        sum += (W)e.coef * Ra[e.a * stride] * Rb[e.b * stride] * Rc[e.c * stride];
+    }
+    acc.add(cur, (u128)sum, false);
+}
+
 template <int NP>
 __global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, const CoreProg P, WorkDesc W,
-                                                      const int* __restrict__ sup, const Sink S) {
-    // program table in shared memory: k | l << 8 | m << 16 | pattern << 24
+                                                      const int* __restrict__ sup, const EdgeTerms T,
+                                                      const Sink S) {
+    extern __shared__ u128 s_rows[];                 // [row entry][thread] (table path)
+    // program table (checked fallback path): k | l << 8 | m << 16 | pattern << 24
     __shared__ uint32_t s_prog[FSGC_MAXPROG];
-    __shared__ int s_kmax, s_minm;
-    __shared__ uint64_t s_venn[8][32][3];            // per warp: the roots' Venn entries
+    __shared__ uint32_t s_q[8][64][3];               // per warp: queued roots (nu, nv, nuv)
+    __shared__ int s_minm;
     if (threadIdx.x == 0) {
-        int kmax = 0, minm = 255;
-        for (int pi = 0; pi < P.nprog; ++pi) {
-            kmax = max(kmax, (int)P.prog[pi].ksum);
-            minm = min(minm, (int)P.em[pi]);
-        }
-        s_kmax = kmax;
+        int minm = 255;
+        for (int pi = 0; pi < P.nprog; ++pi) minm = min(minm, (int)P.em[pi]);
         s_minm = minm;
     }
     if (threadIdx.x < P.nprog)
         s_prog[threadIdx.x] = P.ek[threadIdx.x] | (P.el[threadIdx.x] << 8) | (P.em[threadIdx.x] << 16) |
                               ((uint32_t)P.prog[threadIdx.x].pat << 24);
     __syncthreads();
-    const int nprog = P.nprog, Kmax = s_kmax;
-    const uint64_t minm = (uint64_t)s_minm;
-    const int lane = threadIdx.x & 31;
+    const int nprog = P.nprog;
+    const int minm = s_minm;
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+    const int stride = blockDim.x;
     AccN<NP> acc;
     acc.init();
     unsigned long long nmatch = 0;
+    int cnt = 0;                                      // queue length (warp-uniform)
+
+    // lanes < take each evaluate one queued root, then the rest moves up
+    auto drain = [&](int take) {
+        __syncwarp();
+        if (lane < take) {
+            const uint64_t nu = s_q[wib][lane][0], nv = s_q[wib][lane][1], nuv = s_q[wib][lane][2];
+            const int nbits = T.n > 0 ? bitlen64(nu + nv + nuv) * T.kmax : 1 << 20;
+            if (nbits <= 63) {
+                edge_terms_eval<uint64_t>(nu, nv, nuv, T, (uint64_t*)s_rows + threadIdx.x, stride, acc);
+            } else if (nbits <= 127) {
+                edge_terms_eval<u128>(nu, nv, nuv, T, (u128*)s_rows + threadIdx.x, stride, acc);
+            } else {
+                for (int pi = 0; pi < nprog; ++pi) {
+                    const uint32_t w = s_prog[pi];
+                    bool o = false;
+                    const u128 f = edge_prog_eval(nu, nv, nuv, w, false, o);
+                    acc.add((int)(w >> 24), f, o);
+                }
+            }
+        }
+        __syncwarp();
+        const int rest = cnt - take;
+        if (lane < rest) {
+#pragma unroll
+            for (int x = 0; x < 3; ++x) s_q[wib][lane][x] = s_q[wib][take + lane][x];
+        }
+        cnt = rest;
+        __syncwarp();
+    };
+
     const int64_t total = W.end - W.begin;
     // this shard owns the 32-item chunks g = c * nshards + shard; its items are
-    // numbered L = c * 32 + lane and walked grid-stride, kEdgeILP at a time:
-    // a lane's items lie far apart, so the heavy roots (highest ids, at the
-    // end) are spread over many lanes instead of piling up in one
+    // numbered L = c * 32 + lane and walked grid-stride, kEdgeILP at a time,
+    // transposed (lane l of warp w takes local item l * NW + w of each slice)
+    // so the hub roots (clustered at the end of the degree order) spread out
     const int64_t nchunks = (total + 31) / 32;
     const int64_t mychunks = nchunks > W.shard ? (nchunks - W.shard + W.nshards - 1) / W.nshards : 0;
     const int64_t nloc = mychunks * 32;
     const int64_t nthreads = (int64_t)gridDim.x * blockDim.x;
-    const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
-    const int64_t warp = tid >> 5;
-    const int wib = threadIdx.x >> 5;
+    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
     const bool oriented = P.root_mode == ROOT_ORIENTED;
-    const unsigned long long t_start = W.trace ? gtimer() : 0;
-    unsigned long long tp1 = 0, tp2 = 0, tp3 = 0;
-    int nch = 0;
-    // transposed assignment: lane l of warp w takes local item l * NW + w of
-    // each NT-slice, so the hub roots (clustered at the end of the degree-
-    // ordered list) spread over all warps instead of filling a few
     const int64_t NW = nthreads >> 5;
     const int64_t tpos = (int64_t)lane * NW + warp;
     for (int64_t L0 = 0; L0 < nloc; L0 += nthreads * kEdgeILP) {
-        ++nch;
-        int u[kEdgeILP], v[kEdgeILP];
-        int64_t e[kEdgeILP], itm[kEdgeILP];
+        int u[kEdgeILP], v[kEdgeILP], c[kEdgeILP];
+        int64_t itm[kEdgeILP];
         bool ok[kEdgeILP];
 #pragma unroll
-        for (int j = 0; j < kEdgeILP; ++j) {           // 1: root edges
+        for (int j = 0; j < kEdgeILP; ++j) {           // 1: root edges (+ support, coalesced)
             const int64_t L = L0 + j * nthreads + tpos;
             const int64_t t = ((L >> 5) * W.nshards + W.shard) * 32 + (L & 31);
             ok[j] = L < nloc && t < total;
             itm[j] = W.begin + (ok[j] ? t : 0);
-            if (oriented) { u[j] = __ldg(G.osrc + itm[j]); v[j] = __ldg(G.odst + itm[j]); e[j] = itm[j]; }
-            else { u[j] = __ldg(G.row + itm[j]); v[j] = __ldg(G.adj + itm[j]); }
+            if (oriented) {
+                u[j] = __ldg(G.osrc + itm[j]); v[j] = __ldg(G.odst + itm[j]);
+                c[j] = __ldg(sup + itm[j]);
+            } else {
+                u[j] = __ldg(G.row + itm[j]); v[j] = __ldg(G.adj + itm[j]);
+            }
         }
-        if (W.trace && nch == 1) { __syncwarp(); int z = u[0] + u[kEdgeILP - 1]; if (z == -7) nmatch++; tp1 = gtimer(); }
-        int du[kEdgeILP], dv[kEdgeILP], c[kEdgeILP];
+        if (!oriented) {
 #pragma unroll
-        for (int j = 0; j < kEdgeILP; ++j) {           // 2: degrees + support
-            if (!oriented) e[j] = edge_of_entry(G, O, u[j], v[j], itm[j]);
-            du[j] = (int)(__ldg(G.offs + u[j] + 1) - __ldg(G.offs + u[j]));
-            dv[j] = (int)(__ldg(G.offs + v[j] + 1) - __ldg(G.offs + v[j]));
-            c[j] = __ldg(sup + e[j]);
+            for (int j = 0; j < kEdgeILP; ++j) c[j] = __ldg(sup + edge_of_entry(G, O, u[j], v[j], itm[j]));
+        }
+        int du[kEdgeILP], dv[kEdgeILP];
+#pragma unroll
+        for (int j = 0; j < kEdgeILP; ++j) {           // 2: degrees, only where a program can match
+            du[j] = dv[j] = 0;
+            if (ok[j] && (c[j] >= minm || !W.degfilter)) {
+                du[j] = (int)(__ldg(G.offs + u[j] + 1) - __ldg(G.offs + u[j]));
+                dv[j] = (int)(__ldg(G.offs + v[j] + 1) - __ldg(G.offs + v[j]));
+            }
         }
 #pragma unroll
-        if (W.trace && nch == 1) { int z = c[0] + du[kEdgeILP - 1] + dv[0]; if (z == -7) nmatch++; tp2 = gtimer(); }
-        for (int j = 0; j < kEdgeILP; ++j) {           // 3: Venn diagrams
+        for (int j = 0; j < kEdgeILP; ++j) {           // 3: Venn diagrams -> warp queue
             bool work = false;
-            uint64_t nu = 0, nv = 0, cc = 0;
-            if (ok[j] && !(W.degfilter && (du[j] < P.mindeg[0] || dv[j] < P.mindeg[1]))) {
-                ++nmatch;
-                cc = (uint64_t)c[j];
-                work = cc >= minm;                      // every program needs >= minm wedge fringes
-                nu = du[j] - 1 - cc;
-                nv = dv[j] - 1 - cc;
+            if (ok[j]) {
+                const bool pass = !W.degfilter || (c[j] >= minm && du[j] >= P.mindeg[0] && dv[j] >= P.mindeg[1]);
+                if (pass) ++nmatch;
+                work = pass && c[j] >= minm;           // every program needs >= minm wedge fringes
             }
-            // 4: fc over (root, program) pairs spread across the warp, so a
-            // root with a long program list does not serialise on one lane
             const unsigned wm = __ballot_sync(FULLMASK, work);
-            if (!wm) continue;
             if (work) {
-                s_venn[wib][lane][0] = nu;
-                s_venn[wib][lane][1] = nv;
-                s_venn[wib][lane][2] = cc;
+                const int slot = cnt + __popc(wm & ((1u << lane) - 1));
+                s_q[wib][slot][0] = (uint32_t)(du[j] - 1 - c[j]);
+                s_q[wib][slot][1] = (uint32_t)(dv[j] - 1 - c[j]);
+                s_q[wib][slot][2] = (uint32_t)c[j];
             }
-            __syncwarp();
-            const int total_pairs = __popc(wm) * nprog;
-            for (int t = lane; t < total_pairs; t += 32) {
-                const int k = t / nprog, pi = t - k * nprog;
-                const int src = __fns(wm, 0, k + 1);    // k-th root with work
-                const uint64_t a = s_venn[wib][src][0], b = s_venn[wib][src][1], x = s_venn[wib][src][2];
-                const uint32_t w = s_prog[pi];
-                bool o = false;
-                const u128 f = edge_prog_eval(a, b, x, w, fits64(a + b + x, Kmax), o);
-                acc.add((int)(w >> 24), f, o);
-            }
-            __syncwarp();
+            cnt += __popc(wm);
+            if (cnt >= 32) drain(32);
         }
     }
-    tp3 = W.trace ? gtimer() : 0;
+    if (cnt) drain(cnt);
     block_publish<NP>(acc, nmatch, S);
-    if (W.trace && lane == 0) {
-        unsigned smid;
-        asm volatile("mov.u32 %0, %smid;" : "=r"(smid));
-        unsigned long long* tr = W.trace + 8 * warp;
-        tr[0] = t_start; tr[1] = gtimer(); tr[2] = smid; tr[3] = (unsigned long long)nch;
-        tr[4] = tp1; tr[5] = tp2; tr[6] = tp3;
-    }
 }
 
 // ------------------------------------------------------------------------
@@ -1321,6 +1400,23 @@ static int ensure_binom_table(int dev) {
     if (ready.count(dev)) return FSGC_OK;
     binom_table_init<<<1, 32>>>();
     FSGC_CUDA(cudaGetLastError());
+    {   // inverses of the odd parts of 1..63 mod 2^128 (Newton iteration)
+        uint64_t inv[64] = {0}, invh[64] = {0};
+        uint32_t tz[64] = {0};
+        for (int t = 1; t < 64; ++t) {
+            int z = 0;
+            while (!((t >> z) & 1)) ++z;
+            const u128 od = (u128)(t >> z);
+            u128 x = od;
+            for (int it = 0; it < 7; ++it) x *= (u128)2 - od * x;   // 3 -> 6 -> ... -> 384 correct bits
+            inv[t] = u128_lo(x);
+            invh[t] = u128_hi(x);
+            tz[t] = (uint32_t)z;
+        }
+        FSGC_CUDA(cudaMemcpyToSymbol(c_inv_odd, inv, sizeof inv));
+        FSGC_CUDA(cudaMemcpyToSymbol(c_inv_odd_hi, invh, sizeof invh));
+        FSGC_CUDA(cudaMemcpyToSymbol(c_tz, tz, sizeof tz));
+    }
     FSGC_CUDA(cudaDeviceSynchronize());
     ready.insert(dev);
     return FSGC_OK;
@@ -1340,8 +1436,60 @@ struct PassExec {
     size_t ws_off = 0, sup_bytes = 0, parts_off = 0, bytes = 0;
     int term_base = 0;         // index of this pass's programs in the term offset/count arrays
     bool whole = true;
+    EdgeTerms et{};            // edge cores: the Sec. 3.1 term table (et.n == 0: checked path)
+    size_t smem_fc = 0;        // dynamic shared memory of edge_fc_kernel
 };
+
+// the term table of an edge-core pass (see EdgeTerms); et.n = 0 when a
+// coefficient, the row length or the number of terms exceeds the table limits
+static void build_edge_terms(const CoreProg& cp, EdgeTerms* et) {
+    std::memset(et, 0, sizeof *et);
+    std::map<std::tuple<int, int, int, int>, u128> acc;   // (pat, a, b, c) -> coef
+    int ka = 0, kb = 0, kc = 0, kmax = 0;
+    auto fact = [](int x) { u128 f = 1; for (int i = 2; i <= x; ++i) f *= (u128)i; return f; };
+    for (int pi = 0; pi < cp.nprog; ++pi) {
+        const int k = cp.ek[pi], l = cp.el[pi], m = cp.em[pi];
+        if (k + l + m > 30) return;                       // (i+j+m)! must fit 128 bits
+        kmax = std::max(kmax, (int)cp.prog[pi].ksum);
+        for (int i = 0; i <= k; ++i)
+            for (int j = 0; j <= l; ++j) {
+                const u128 coef = fact(i + j + m) / (fact(i) * fact(j) * fact(m));
+                acc[std::make_tuple((int)cp.prog[pi].pat, k - i, l - j, i + j + m)] += coef;
+                ka = std::max(ka, k - i);
+                kb = std::max(kb, l - j);
+                kc = std::max(kc, i + j + m);
+            }
+    }
+    if ((int)acc.size() > kMaxEdgeTerms || ka + kb + kc + 3 > kMaxRowEntries || kmax > 63) return;
+    int n = 0;
+    for (auto& kv : acc) {   // ordered by pattern
+        if (kv.second >> 63) return;
+        EdgeTerm& t = et->t[n++];
+        t.pat = (uint8_t)std::get<0>(kv.first);
+        t.a = (uint8_t)std::get<1>(kv.first);
+        t.b = (uint8_t)std::get<2>(kv.first);
+        t.c = (uint8_t)std::get<3>(kv.first);
+        t.coef = (uint64_t)kv.second;
+    }
+    et->n = n;
+    et->ka = ka; et->kb = kb; et->kc = kc;
+    et->kmax = kmax;
+}
 }  // namespace
+
+// device copies of the partition-lattice term tables of a pattern batch;
+// graph independent, so cached per (device, patterns) -- a new graph with the
+// same patterns (e2e: load + count every step) allocates nothing here
+struct DevTerms {
+    PartTerm* terms = nullptr;
+    int32_t* off = nullptr;
+    int32_t* cnt = nullptr;
+    ~DevTerms() {
+        if (terms) cudaFree(terms);
+        if (off) cudaFree(off);
+        if (cnt) cudaFree(cnt);
+    }
+};
 
 struct fsgc_plan {
     const fsgc_graph* g = nullptr;
@@ -1352,15 +1500,10 @@ struct fsgc_plan {
     int device = 0;
     std::vector<cudaEvent_t> ev;   // 3 per pass
     unsigned long long* trace = nullptr;
-    PartTerm* terms_dev = nullptr;   // partition-lattice terms of all programs
-    int32_t* off_dev = nullptr;
-    int32_t* cnt_dev = nullptr;
+    std::shared_ptr<DevTerms> terms;   // partition-lattice terms of all programs
     ~fsgc_plan() {
         for (auto e : ev) cudaEventDestroy(e);
         if (trace) cudaFree(trace);
-        if (terms_dev) cudaFree(terms_dev);
-        if (off_dev) cudaFree(off_dev);
-        if (cnt_dev) cudaFree(cnt_dev);
     }
 };
 
@@ -1420,7 +1563,10 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
                                                                 (g->m + 255) / 256));
             int64_t mine = ((e - b) + 31) / 32;
             mine = (mine + opts.shard_count - 1) / opts.shard_count;
-            X.grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy(kernel_for(1, X.npc), 256, 0),
+            build_edge_terms(cp, &X.et);
+            if (tune("FSGC_NO_EDGE_TERMS", 0)) X.et.n = 0;
+            X.smem_fc = X.et.n ? (size_t)(X.et.ka + X.et.kb + X.et.kc + 3) * 256 * sizeof(u128) : 0;
+            X.grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy(kernel_for(1, X.npc), 256, X.smem_fc),
                                                             (mine + 7) / 8));
             if (tune("FSGC_EDGE_BLOCKS", 0) > 0) X.grid = tune("FSGC_EDGE_BLOCKS", 0);
             X.sup_bytes = (size_t)std::max<int64_t>(g->m, 1) * sizeof(int);
@@ -1447,7 +1593,13 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
         P->passes.push_back(X);
     }
     P->ws_bytes = off;
-    {   // partition-lattice term tables -> device
+    {   // partition-lattice term tables -> device (cached)
+        static std::mutex tmu;
+        static std::map<std::vector<uint64_t>, std::shared_ptr<DevTerms>> tcache;
+        std::vector<uint64_t> tkey{(uint64_t)dev, (uint64_t)opts.no_symmetry_breaking};
+        for (int i = 0; i < npats; ++i) tkey.push_back(pats[i]->uid);
+        std::lock_guard<std::mutex> lock(tmu);
+        auto it = tcache.find(tkey);
         std::vector<PartTerm> all;
         std::vector<int32_t> offs, cnts;
         for (auto& X : P->passes) {
@@ -1459,14 +1611,22 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
                 all.insert(all.end(), T.begin(), T.end());
             }
         }
-        if (all.empty()) all.push_back(PartTerm{});
-        if (offs.empty()) { offs.push_back(0); cnts.push_back(-1); }
-        FSGC_CUDA(cudaMalloc(&P->terms_dev, all.size() * sizeof(PartTerm)));
-        FSGC_CUDA(cudaMalloc(&P->off_dev, offs.size() * sizeof(int32_t)));
-        FSGC_CUDA(cudaMalloc(&P->cnt_dev, cnts.size() * sizeof(int32_t)));
-        FSGC_CUDA(cudaMemcpy(P->terms_dev, all.data(), all.size() * sizeof(PartTerm), cudaMemcpyHostToDevice));
-        FSGC_CUDA(cudaMemcpy(P->off_dev, offs.data(), offs.size() * sizeof(int32_t), cudaMemcpyHostToDevice));
-        FSGC_CUDA(cudaMemcpy(P->cnt_dev, cnts.data(), cnts.size() * sizeof(int32_t), cudaMemcpyHostToDevice));
+        if (it != tcache.end()) {
+            P->terms = it->second;
+        } else {
+            if (all.empty()) all.push_back(PartTerm{});
+            if (offs.empty()) { offs.push_back(0); cnts.push_back(-1); }
+            std::shared_ptr<DevTerms> T(new DevTerms);
+            FSGC_CUDA(cudaMalloc(&T->terms, all.size() * sizeof(PartTerm)));
+            FSGC_CUDA(cudaMalloc(&T->off, offs.size() * sizeof(int32_t)));
+            FSGC_CUDA(cudaMalloc(&T->cnt, cnts.size() * sizeof(int32_t)));
+            FSGC_CUDA(cudaMemcpy(T->terms, all.data(), all.size() * sizeof(PartTerm), cudaMemcpyHostToDevice));
+            FSGC_CUDA(cudaMemcpy(T->off, offs.data(), offs.size() * sizeof(int32_t), cudaMemcpyHostToDevice));
+            FSGC_CUDA(cudaMemcpy(T->cnt, cnts.data(), cnts.size() * sizeof(int32_t), cudaMemcpyHostToDevice));
+            if (tcache.size() > 256) tcache.clear();
+            tcache[tkey] = T;
+            P->terms = T;
+        }
     }
     P->ev.resize(3 * P->passes.size());
     for (auto& ev : P->ev) FSGC_CUDA(cudaEventCreate(&ev));
@@ -1502,16 +1662,14 @@ extern "C" int fsgc_plan_enqueue(const fsgc_plan* P, void* workspace, void* raw_
         AccDev* dacc = (AccDev*)base;
         unsigned long long* dmatch = (unsigned long long*)(base + sizeof(AccDev) * FSGC_MAXPATS);
         unsigned long long* dqueue = dmatch + 1;
-        unsigned long long* dqueue2 = dmatch + 2;
         unsigned int* dticket = (unsigned int*)(dmatch + 3);
         int* dsup = (int*)(base + kHdrBytes);
         Sink S{dacc, dmatch, (BlockPartial*)(base + X.parts_off), dticket, P->publish_mode};
         WorkDesc W = X.W;
-        if (P->trace && X.kind == 1) W.trace = P->trace;
         const CoreProg& cp = X.plan.prog;
         FSGC_CUDA(cudaEventRecordWithFlags(P->ev[3 * pi], st, evflags));
         if (X.kind != 0 && g->m > 0) {   // (A) per-edge common-neighbour counts
-            support_kernel<<<(int)X.grid_sup, 256, 0, st>>>(G, O, g->m, dsup, dqueue2,
+            support_kernel<<<(int)X.grid_sup, 256, 0, st>>>(G, O, g->m, dsup, g->sorder, g->ssrc, g->sdst,
                                                              P->trace ? P->trace + (1 << 17) : nullptr);
             FSGC_CUDA(cudaGetLastError());
         }
@@ -1519,16 +1677,16 @@ extern "C" int fsgc_plan_enqueue(const fsgc_plan* P, void* workspace, void* raw_
         if (W.end > W.begin) {
             const void* fn = kernel_for(X.kind, X.npc);
             void* args_v[] = {(void*)&G, (void*)&cp, (void*)&W, (void*)&S};
-            void* args_e[] = {(void*)&G, (void*)&O, (void*)&cp, (void*)&W, (void*)&dsup, (void*)&S};
+            void* args_e[] = {(void*)&G, (void*)&O, (void*)&cp, (void*)&W, (void*)&dsup, (void*)&X.et, (void*)&S};
             HubDev Hd{g->hub_base, g->hub_words, g->hub_bits};
-            TermDev TD{P->terms_dev, P->off_dev + X.term_base, P->cnt_dev + X.term_base};
+            TermDev TD{P->terms->terms, P->terms->off + X.term_base, P->terms->cnt + X.term_base};
             void* args_c[] = {(void*)&G, (void*)&O, (void*)&Hd, (void*)&cp, (void*)&W, (void*)&dsup, (void*)&TD,
                               (void*)&S, (void*)&dqueue};
             void* args_t[] = {(void*)&G, (void*)&O, (void*)&Hd, (void*)&cp, (void*)&W, (void*)&dsup, (void*)&S};
             if (X.kind == 0)
                 FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(256), args_v, 0, st));
             else if (X.kind == 1)    // (B) fringe counts per root edge
-                FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(256), args_e, 0, st));
+                FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(256), args_e, X.smem_fc, st));
             else if (X.kind == 3)
                 FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(kTriWarps * 32), args_t, 0, st));
             else

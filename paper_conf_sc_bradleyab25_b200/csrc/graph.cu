@@ -142,6 +142,50 @@ struct UpperTri {
     __host__ __device__ bool operator()(const uint64_t& k) const { return (k >> B) < (k & mask); }
 };
 
+// support-pass work order: key = merge length out(u) + out(v) of oriented
+// edge i (capped), value = i; sorted, so the 32 lanes of a warp get roots of
+// similar cost (degree-aware binning, north_star)
+__global__ void support_work_keys(const int64_t* __restrict__ offs, const int64_t* __restrict__ split,
+                                  const int32_t* __restrict__ osrc, const int32_t* __restrict__ odst, int64_t m,
+                                  uint32_t* __restrict__ key, int32_t* __restrict__ idx) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        const int u = osrc[i], v = odst[i];
+        const int64_t w = (offs[u + 1] - split[u]) + (offs[v + 1] - split[v]);
+        key[i] = (uint32_t)(w < (1 << 20) ? w : (1 << 20) - 1);
+        idx[i] = (int32_t)i;
+    }
+}
+
+__global__ void gather_uv(const int32_t* __restrict__ idx, const int32_t* __restrict__ osrc,
+                          const int32_t* __restrict__ odst, int64_t m, int32_t* __restrict__ su,
+                          int32_t* __restrict__ sv) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m;
+         i += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t e = idx[i];
+        su[i] = osrc[e];
+        sv[i] = odst[e];
+    }
+}
+
+// number of unique keys without the trailing sentinel run (dnum[0] in, out)
+__global__ void unique_count(const uint64_t* __restrict__ uniq, int64_t* dnum, uint64_t sentinel) {
+    const int64_t nu = dnum[0];
+    dnum[0] = (nu > 0 && uniq[nu - 1] == sentinel) ? nu - 1 : nu;
+}
+
+// out[0] = first v in [lo, n) with deg(v) >= mindeg (n if none), out[1] = deg(n-1)
+__global__ void hub_search(const int64_t* __restrict__ offs, int64_t n, int64_t lo, int64_t mindeg,
+                           int64_t* out) {
+    int64_t hi = n;
+    while (lo < hi) {
+        const int64_t mid = (lo + hi) >> 1;
+        if (offs[mid + 1] - offs[mid] >= mindeg) hi = mid; else lo = mid + 1;
+    }
+    out[0] = lo;
+    out[1] = offs[n] - offs[n - 1];
+}
+
 int grid_for(int64_t work) {
     int64_t g = (work + 255) / 256;
     if (g > 148 * 32) g = 148 * 32;
@@ -192,7 +236,7 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
     DevBuf<char> tmp;
     size_t tmp_bytes = 0;
     DevBuf<int64_t> dnum;
-    FSGC_CUDA(dnum.alloc(1, st));
+    FSGC_CUDA(dnum.alloc(2, st));
     int64_t M = 0;
     if (K > 0) {
         cub::DoubleBuffer<uint64_t> db(ka.ptr, kb.ptr);
@@ -205,20 +249,16 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
         FSGC_CUDA(cub::DeviceSelect::Unique(nullptr, ub, sorted, other, dnum.ptr, K, st));
         if (ub > tmp_bytes) { FSGC_CUDA(tmp.alloc(ub, st)); tmp_bytes = ub; }
         FSGC_CUDA(cub::DeviceSelect::Unique(tmp.ptr, ub, sorted, other, dnum.ptr, K, st));
-        int64_t nu = 0;
-        uint64_t last = 0;
-        FSGC_CUDA(cudaMemcpyAsync(&nu, dnum.ptr, sizeof nu, cudaMemcpyDeviceToHost, st));
-        FSGC_CUDA(cudaStreamSynchronize(st));
-        if (nu > 0) {
-            FSGC_CUDA(cudaMemcpyAsync(&last, other + nu - 1, sizeof last, cudaMemcpyDeviceToHost, st));
-            FSGC_CUDA(cudaStreamSynchronize(st));
-        }
-        M = (nu > 0 && last == sentinel) ? nu - 1 : nu;
+        unique_count<<<1, 1, 0, st>>>(other, dnum.ptr, sentinel);   // drop the sentinel run
+        FSGC_CUDA(cudaGetLastError());
         if (other != ka.ptr) std::swap(ka.ptr, kb.ptr);  // unique keys now in ka
     }
-    int bad = 0;
-    FSGC_CUDA(cudaMemcpyAsync(&bad, dbad.ptr, sizeof bad, cudaMemcpyDeviceToHost, st));
+    int64_t hv[2] = {0, 0};   // M, bad flag: one host synchronisation
+    FSGC_CUDA(cudaMemcpyAsync(&hv[0], dnum.ptr, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+    FSGC_CUDA(cudaMemcpyAsync(&hv[1], dbad.ptr, sizeof(int), cudaMemcpyDeviceToHost, st));
     FSGC_CUDA(cudaStreamSynchronize(st));
+    if (K > 0) M = hv[0];
+    const int bad = (int)hv[1];
     if (bad) FSGC_FAIL(FSGC_ERR_INVALID, "edge list contains a vertex id outside [0, %lld)", (long long)n);
     kb.release();
 
@@ -306,6 +346,29 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
         if (b > tmp_bytes) { FSGC_CUDA(tmp.alloc(b, st)); tmp_bytes = b; }
         FSGC_CUDA(cub::DeviceScan::ExclusiveSum(tmp.ptr, b, oofs.ptr, oofs.ptr, n + 1, st));
     }
+    // support-pass order (sorted by merge length) with its (u, v) gathered
+    DevBuf<int32_t> sorder, ssrc, sdst;
+    if (m > 0) {
+        DevBuf<uint32_t> k0, k1;
+        DevBuf<int32_t> i1;
+        FSGC_CUDA(k0.alloc(m, st));
+        FSGC_CUDA(k1.alloc(m, st));
+        FSGC_CUDA(sorder.alloc(m, st));
+        FSGC_CUDA(i1.alloc(m, st));
+        support_work_keys<<<grid_for(m), 256, 0, st>>>(offs.ptr, split.ptr, osrc.ptr, odst.ptr, m, k0.ptr, sorder.ptr);
+        FSGC_CUDA(cudaGetLastError());
+        cub::DoubleBuffer<uint32_t> dk(k0.ptr, k1.ptr);
+        cub::DoubleBuffer<int32_t> dv(sorder.ptr, i1.ptr);
+        size_t b = 0;
+        FSGC_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, b, dk, dv, m, 0, 20, st));
+        if (b > tmp_bytes) { FSGC_CUDA(tmp.alloc(b, st)); tmp_bytes = b; }
+        FSGC_CUDA(cub::DeviceRadixSort::SortPairs(tmp.ptr, b, dk, dv, m, 0, 20, st));
+        if (dv.Current() != sorder.ptr) std::swap(sorder.ptr, i1.ptr);
+        FSGC_CUDA(ssrc.alloc(m, st));
+        FSGC_CUDA(sdst.alloc(m, st));
+        gather_uv<<<grid_for(m), 256, 0, st>>>(sorder.ptr, osrc.ptr, odst.ptr, m, ssrc.ptr, sdst.ptr);
+        FSGC_CUDA(cudaGetLastError());
+    }
     tmp.release();
     ka.release();
     kb.release();
@@ -314,6 +377,7 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
     // hub bitmaps within a memory budget (default min(4 GiB, 5% of device
     // memory); FSGC_HUB_BYTES overrides), only for degree >= kHubMinDeg
     int64_t hub_base = n, hub_words = (n + 31) / 32;
+    int64_t maxdeg = 0;   // the last vertex has the largest degree
     DevBuf<uint32_t> hubs;
     {
         size_t free_b = 0, total_b = 0;
@@ -324,31 +388,24 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
         const int64_t per = hub_words * 4;
         int64_t max_hubs = per > 0 ? budget / per : 0;
         if (max_hubs > n) max_hubs = n;
-        if (max_hubs > 0 && M > 0) {
-            // smallest candidate base: the max_hubs highest ids; raise it until deg >= threshold
-            int64_t lo = n - max_hubs, hi = n;   // find first v in [lo, n) with deg(v) >= kHubMinDeg
-            const int64_t kHubMinDeg = 256;
-            while (lo < hi) {
-                int64_t mid = (lo + hi) / 2;
-                int64_t o2[2];
-                FSGC_CUDA(cudaMemcpy(o2, offs.ptr + mid, 2 * sizeof(int64_t), cudaMemcpyDeviceToHost));
-                if (o2[1] - o2[0] >= kHubMinDeg) hi = mid; else lo = mid + 1;
-            }
-            hub_base = lo;
+        // first v in [n - max_hubs, n) with deg(v) >= kHubMinDeg (degrees are
+        // ascending in the new ids), and the maximum degree: one synchronisation
+        int64_t hv2[2] = {n, 0};
+        if (n > 0) {
+            hub_search<<<1, 1, 0, st>>>(offs.ptr, n, n - std::max<int64_t>(0, std::min<int64_t>(max_hubs, n)),
+                                        M > 0 ? 256 : (int64_t)1 << 62, dnum.ptr);
+            FSGC_CUDA(cudaGetLastError());
+            FSGC_CUDA(cudaMemcpyAsync(hv2, dnum.ptr, 2 * sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+            FSGC_CUDA(cudaStreamSynchronize(st));
         }
+        if (max_hubs > 0 && M > 0) hub_base = hv2[0];
+        maxdeg = hv2[1];
         if (hub_base < n) {
             FSGC_CUDA(hubs.alloc((size_t)(n - hub_base) * hub_words, st));
             FSGC_CUDA(cudaMemsetAsync(hubs.ptr, 0, (size_t)(n - hub_base) * hub_words * 4, st));
             hub_bitmaps<<<grid_for(M), 256, 0, st>>>(offs.ptr, adj.ptr, hub_base, n, hub_words, hubs.ptr);
             FSGC_CUDA(cudaGetLastError());
         }
-    }
-    int64_t maxdeg = 0;
-    if (n > 0) {
-        int64_t lastoffs[2] = {0, 0};
-        FSGC_CUDA(cudaMemcpyAsync(lastoffs, offs.ptr + n - 1, 2 * sizeof(int64_t), cudaMemcpyDeviceToHost, st));
-        FSGC_CUDA(cudaStreamSynchronize(st));
-        maxdeg = lastoffs[1] - lastoffs[0];  // the last vertex has the largest degree
     }
     FSGC_CUDA(cudaStreamSynchronize(st));
 
@@ -366,6 +423,9 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
     g->order = order.take();
     g->split = split.take();
     g->oofs = oofs.take();
+    g->sorder = sorder.take();
+    g->ssrc = ssrc.take();
+    g->sdst = sdst.take();
     g->hub_base = hub_base;
     g->hub_words = hub_words;
     g->hub_bits = hubs.take();
@@ -406,6 +466,9 @@ extern "C" void fsgc_free_graph(fsgc_graph* g) {
     cudaFree(g->order);
     cudaFree(g->split);
     cudaFree(g->oofs);
+    cudaFree(g->sorder);
+    cudaFree(g->ssrc);
+    cudaFree(g->sdst);
     cudaFree(g->hub_bits);
     delete g;
 }

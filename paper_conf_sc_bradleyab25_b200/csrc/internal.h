@@ -29,6 +29,11 @@ struct fsgc_graph {
     int64_t* oofs = nullptr;     // [n+1] oriented offsets: oriented index of
                                  //       CSR position p >= split[u] is
                                  //       oofs[u] + p - split[u]
+    // support-pass work order: oriented edge ids sorted by out(u) + out(v),
+    // with their endpoints (coalesced reads in that order)
+    int32_t* sorder = nullptr;   // [m]
+    int32_t* ssrc = nullptr;     // [m]
+    int32_t* sdst = nullptr;     // [m]
     // hub bitmaps: vertices v >= hub_base (the highest-degree ones, ids are
     // degree ordered) have a dense n-bit adjacency bitmap (O(1) membership)
     int64_t hub_base = 0;        // == n when there are no hubs

@@ -267,3 +267,45 @@ def test_triangle_core_kernel_with_hub_bitmaps(monkeypatch):
         assert x.count == y.count == z.count, P.name
     for P, x in zip(pats[:2], a[:2]):
         assert x.count == oracle.fringe_count(gadj, P.n, P.edges, P.core), P.name
+
+
+def _edge_core_pattern(k, l, m):
+    """edge core {0,1}: k tails on 0, l tails on 1, m wedge fringes (Sec. 3.1)."""
+    from inputs.patterns import _p
+    e = [(0, 1)]
+    nxt = 2
+    for _ in range(k):
+        e.append((0, nxt)); nxt += 1
+    for _ in range(l):
+        e.append((1, nxt)); nxt += 1
+    for _ in range(m):
+        e += [(0, nxt), (1, nxt)]; nxt += 1
+    return _p(f"edge+{k}t{l}t{m}w", nxt, e)
+
+
+def test_edge_core_counts_beyond_64_bits():
+    """Two adjacent hubs with 1,200 / 1,000 private leaves and 20 common
+    neighbours: edge-core counts with up to 15 fringes exceed 2^64.  The bench
+    kernel's three arithmetic tiers all run: 64-bit term table (leaf edges),
+    128-bit term table (N^K < 2^127), checked per-program 128-bit (15 fringes
+    on the hub edge).  vs the oracle."""
+    A, B = 0, 1
+    e = [(A, B)]
+    nxt = 2
+    for _ in range(1200):
+        e.append((A, nxt)); nxt += 1
+    for _ in range(1000):
+        e.append((B, nxt)); nxt += 1
+    for _ in range(20):
+        e += [(A, nxt), (B, nxt)]; nxt += 1
+    for i in range(2, 200, 2):                        # a few leaf-leaf edges
+        e.append((i, i + 1))
+    n = nxt
+    e = np.array(e, dtype=np.int64)
+    _, _, _, gadj = oracle_graph(n, e)
+    pats = [_edge_core_pattern(*x) for x in [(6, 4, 0), (8, 0, 1), (3, 3, 3), (5, 5, 0), (1, 0, 1), (2, 1, 2), (10, 5, 0)]]
+    g = F.fsgc_load_graph(e, n)
+    res = F.fsgc_count(g, [F.compile_named(P) for P in pats])
+    assert any(r.count is not None and r.count >= 1 << 64 for r in res)
+    for P, r in zip(pats, res):
+        assert not r.overflow and r.count == oracle.fringe_count(gadj, P.n, P.edges, P.core), P.name
