@@ -1279,7 +1279,13 @@ int occupancy(const void* fn, int threads, size_t smem) {
     auto it = cache.find(key);
     if (it != cache.end()) return it->second;
     int n = 0;
-    if (smem > 48 * 1024) cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    // the opt-in limit only grows (a plan with less shared memory must not
+    // lower it below what an earlier plan of the same kernel launches with)
+    static std::map<const void*, size_t> optin;
+    if (smem > optin[fn]) {   // (static + dynamic above 48 KB needs the opt-in)
+        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        optin[fn] = smem;
+    }
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, threads, smem);
     n = std::max(n, 1);
     cache[key] = n;
