@@ -192,6 +192,15 @@ typedef struct {
  * instance is visited, so fsgc_result.core_matches is the number of core
  * instances in the graph (within the root range) */
 #define FSGC_FLAG_NO_DEGREE_FILTER 1
+/* multi-GPU (north_star "root-edge ranges are sharded"): with shard_count > 1
+ * the per-edge support pass c(e) = |N(u) & N(v)| (the oriented triangle
+ * listing that edge, triangle and general cores read) is sharded too: shard s
+ * lists the triangles of the support-order chunks s, s + shard_count, ...
+ * into a partial array, and the caller SUMS the shards' partial arrays (one
+ * all-reduce of int32[m], fsgc_plan_support_region) between the two stages of
+ * fsgc_plan_enqueue_stage.  Without the flag every shard computes the whole
+ * support array itself (no exchange).  fsgc_count rejects the flag. */
+#define FSGC_FLAG_SHARD_SUPPORT 2
 
 /*
  * fsgc_count -- count npats patterns on graph g in ONE pass over the core
@@ -259,6 +268,25 @@ int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* pats, int n
                      const fsgc_count_opts* opts, fsgc_plan** out);
 int fsgc_plan_workspace_bytes(const fsgc_plan* plan, size_t* ws, size_t* raw);
 int fsgc_plan_enqueue(const fsgc_plan* plan, void* workspace, void* raw_out, void* stream);
+
+/*
+ * Staged enqueue (same rules as fsgc_plan_enqueue; stages is a bit mask):
+ *   FSGC_STAGE_SUPPORT  zero the support array and run the support pass
+ *                       (this shard's part with FSGC_FLAG_SHARD_SUPPORT)
+ *   FSGC_STAGE_COUNT    every pass's counting kernel (reads the support
+ *                       array as it is in the workspace) + the raw copy
+ * fsgc_plan_enqueue == both stages; it fails with FSGC_ERR_INVALID for a
+ * plan whose support pass is sharded.
+ * fsgc_plan_support_region: the support array is int32[*count] at byte
+ * *offset of the workspace (*count = 0: no pass of the plan reads it).  It
+ * is indexed by oriented edge (u < v) in (u, v) order.
+ */
+#define FSGC_STAGE_SUPPORT 1
+#define FSGC_STAGE_COUNT 2
+#define FSGC_STAGE_ALL 3
+int fsgc_plan_enqueue_stage(const fsgc_plan* plan, void* workspace, void* raw_out, int stages,
+                            void* stream);
+int fsgc_plan_support_region(const fsgc_plan* plan, size_t* offset, int64_t* count);
 int fsgc_plan_decode(const fsgc_plan* plan, const void* raw, fsgc_result* results);
 void fsgc_plan_free(fsgc_plan* plan);
 

@@ -21,13 +21,17 @@ FSGC_MAX_CORE = 8
 FSGC_MAX_VENN_BITS = 6
 FSGC_MAX_BATCH = 16
 FSGC_FLAG_NO_DEGREE_FILTER = 1
+FSGC_FLAG_SHARD_SUPPORT = 2
+FSGC_STAGE_SUPPORT = 1
+FSGC_STAGE_COUNT = 2
+FSGC_STAGE_ALL = 3
 
 EXPORTS = [
     "fsgc_load_graph", "fsgc_graph_get_info", "fsgc_graph_download", "fsgc_free_graph",
     "fsgc_compile_pattern", "fsgc_pattern_get_info", "fsgc_free_pattern",
     "fsgc_count", "fsgc_num_roots", "fsgc_finalize", "fsgc_last_error", "fsgc_version",
     "fsgc_plan_create", "fsgc_plan_workspace_bytes", "fsgc_plan_enqueue", "fsgc_plan_decode",
-    "fsgc_plan_free",
+    "fsgc_plan_free", "fsgc_plan_enqueue_stage", "fsgc_plan_support_region",
 ]
 
 
@@ -105,6 +109,8 @@ def _load():
         "fsgc_plan_create": ([vp, vp, C.c_int, C.POINTER(CountOpts), C.POINTER(vp)], C.c_int),
         "fsgc_plan_workspace_bytes": ([vp, C.POINTER(C.c_size_t), C.POINTER(C.c_size_t)], C.c_int),
         "fsgc_plan_enqueue": ([vp, vp, vp, vp], C.c_int),
+        "fsgc_plan_enqueue_stage": ([vp, vp, vp, C.c_int, vp], C.c_int),
+        "fsgc_plan_support_region": ([vp, C.POINTER(C.c_size_t), C.POINTER(i64)], C.c_int),
         "fsgc_plan_decode": ([vp, vp, C.POINTER(Result)], C.c_int),
         "fsgc_plan_free": ([vp], None),
         "fsgc_last_error": ([], C.c_char_p),

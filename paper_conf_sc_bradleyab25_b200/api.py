@@ -162,14 +162,15 @@ def compile_named(p) -> Pattern:
 
 
 def _opts(root_begin=0, root_end=-1, shard_index=0, shard_count=1, no_symmetry_breaking=False,
-          no_degree_filter=False):
+          no_degree_filter=False, shard_support=False):
     o = CountOpts()
     o.root_begin = root_begin
     o.root_end = root_end
     o.shard_index = shard_index
     o.shard_count = shard_count
     o.no_symmetry_breaking = 1 if no_symmetry_breaking else 0
-    o.flags = _lib.FSGC_FLAG_NO_DEGREE_FILTER if no_degree_filter else 0
+    o.flags = ((_lib.FSGC_FLAG_NO_DEGREE_FILTER if no_degree_filter else 0) |
+               (_lib.FSGC_FLAG_SHARD_SUPPORT if shard_support else 0))
     return o
 
 
@@ -223,6 +224,21 @@ class Plan:
     def enqueue(self, stream=None):
         check(lib.fsgc_plan_enqueue(self._h, C.c_void_p(self.workspace.data_ptr()),
                                     C.c_void_p(self.raw.data_ptr()), _stream_handle(stream)))
+
+    def enqueue_stage(self, stages, stream=None):
+        """stages: FSGC_STAGE_SUPPORT | FSGC_STAGE_COUNT bit mask"""
+        check(lib.fsgc_plan_enqueue_stage(self._h, C.c_void_p(self.workspace.data_ptr()),
+                                          C.c_void_p(self.raw.data_ptr()), int(stages),
+                                          _stream_handle(stream)))
+
+    def support(self):
+        """the plan's per-edge support array as an int32 view of the
+        workspace (None when no pass reads it)"""
+        off, cnt = C.c_size_t(), C.c_int64()
+        check(lib.fsgc_plan_support_region(self._h, C.byref(off), C.byref(cnt)))
+        if cnt.value == 0:
+            return None
+        return self.workspace[off.value:off.value + 4 * cnt.value].view(dtype=__import__("torch").int32)
 
     def decode(self) -> List[CountResult]:
         res = (Result * len(self.patterns))()
@@ -301,14 +317,47 @@ def combine_partials(part: Sequence[CountResult], group=None, device=None) -> Li
     return out
 
 
+_dist_plans = {}
+
+
+def distributed_plan(graph: Graph, patterns: Sequence[Pattern], rank: int, world: int, **kw) -> Plan:
+    """cached plan of this rank's shard: root chunks AND the support pass's
+    chunks dealt round-robin (FSGC_FLAG_SHARD_SUPPORT)"""
+    key = (graph.handle.value, tuple(p.handle.value for p in patterns), rank, world,
+           tuple(sorted(kw.items())))
+    plan = _dist_plans.get(key)
+    if plan is None or plan.graph is not graph:
+        if len(_dist_plans) > 64:
+            _dist_plans.clear()
+        plan = Plan(graph, patterns, shard_index=rank, shard_count=world, shard_support=world > 1, **kw)
+        _dist_plans[key] = plan
+    return plan
+
+
 def fsgc_count_distributed(graph: Graph, patterns: Sequence[Pattern], group=None, stream=None,
                            **kw) -> List[CountResult]:
     """Strong-scaling count over the ranks of ``group``: the graph is
-    replicated, root chunks are dealt round-robin (shard = rank), and the
-    per-rank 128-bit partial sums are combined by ONE all-reduce (NCCL over
-    NVLink on CUDA tensors; gloo on CPU tensors)."""
+    replicated in every rank's HBM; the support pass's chunks and the root
+    chunks are dealt round-robin (shard = rank).  Two exchanges:
+      1. the per-edge support array (int32[m], partial triangle counts of
+         each shard) is summed by an all-reduce between the two stages;
+      2. the per-rank 128-bit partial sums are combined by ONE all-reduce.
+    NCCL over NVLink for CUDA tensors; gloo works too (CUDA tensors are
+    staged through the host)."""
+    import torch
     import torch.distributed as dist
     rank = dist.get_rank(group)
     world = dist.get_world_size(group)
-    part = fsgc_count(graph, patterns, stream=stream, shard_index=rank, shard_count=world, **kw)
-    return combine_partials(part, group)
+    if world == 1:
+        return fsgc_count(graph, patterns, stream=stream, **kw)
+    pats = list(patterns)
+    plan = distributed_plan(graph, pats, rank, world, **kw)
+    st = stream if stream is not None else torch.cuda.current_stream()
+    with torch.cuda.stream(st):
+        plan.enqueue_stage(_lib.FSGC_STAGE_SUPPORT, st)
+        sup = plan.support()
+        if sup is not None:
+            dist.all_reduce(sup, group=group)
+        plan.enqueue_stage(_lib.FSGC_STAGE_COUNT, st)
+    st.synchronize()
+    return combine_partials(plan.decode(), group)

@@ -30,6 +30,8 @@
 #include <string>
 #include <cstdlib>
 #include <cstdio>
+#include <cmath>
+#include <functional>
 #include "devbuf.cuh"
 #include "u128.cuh"
 #include "fc.cuh"
@@ -412,16 +414,20 @@ __device__ __forceinline__ int support_warp(const int32_t* __restrict__ adj, con
 __global__ void __launch_bounds__(256) support_kernel(GraphDev G, OrientDev O, int64_t m, int* __restrict__ sup,
                                                       const int32_t* __restrict__ sorder,
                                                       const int32_t* __restrict__ ssrc,
-                                                      const int32_t* __restrict__ sdst,
-                                                      unsigned long long* trace) {
+                                                      const int32_t* __restrict__ sdst, int shard,
+                                                      int nshards, unsigned long long* trace) {
     const int lane = threadIdx.x & 31;
     const unsigned long long t_start = trace ? gtimer() : 0;
     int nch = 0;
     const int64_t NW = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t nchunks = (m + 31) >> 5;
-    for (int64_t ch = warp; ch < nchunks; ch += NW) {
+    // shard s of n takes the 32-root chunks s, s + n, ... (interleaved over
+    // the merge-length order, so every shard gets the same cost mix)
+    const int64_t nchunks = ((m + 31) >> 5) - shard;
+    const int64_t mychunks = nchunks > 0 ? (nchunks + nshards - 1) / nshards : 0;
+    for (int64_t vch = warp; vch < mychunks; vch += NW) {
         ++nch;
+        const int64_t ch = vch * nshards + shard;
         const int64_t t = ch * 32 + lane;
         const bool valid = t < m;
         int64_t e = 0;
@@ -670,6 +676,96 @@ __global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, c
 }
 
 // ------------------------------------------------------------------------
+// Venn term tables (triangle and general cores).  Listing 5 distributes the
+// k_t fringes of every type over the Venn regions r covering its anchor set;
+// with x_{t,r} fringes of type t in region r and s_r = sum_t x_{t,r},
+//   fc = sum_x prod_r C(n_r; x_{1,r}, .., x_{T,r}, n_r - s_r)
+//      = sum_s M(s) prod_r C(n_r, s_r),   M(s) = sum_{x -> s} prod_r s_r! / prod_t x_{t,r}!
+// (the multinomial split of each region).  M depends on the pattern only, so
+// the host enumerates Listing 5's tree ONCE per pass, merging the terms of
+// every program (coset of Aut_C') of a pattern; a core match then costs its
+// binomial rows C(n_r, 0..max s_r) plus one product chain per distinct s --
+// e.g. Fig. 4 on the triangle core: 2,889 terms instead of 6 x 18,000
+// Listing 5 leaves.
+constexpr int kMaxVennTerms = 8192;
+constexpr int kMaxVennRows = 64;
+constexpr int kMaxVennNz = 14;
+struct VTerm {
+    uint64_t coef;
+    uint8_t pat, nz;
+    uint8_t off[kMaxVennNz];     // row entries (base[r] + s_r - 1) of the regions with s_r > 0
+};
+struct VennDev {
+    const VTerm* __restrict__ terms;
+    int32_t n;                   // terms; 0: table off (per-program Listing 5)
+    int32_t nrows;               // row entries per core match (C(n_r, j), j >= 1)
+    float slack;                 // log2(programs per pattern) + margin
+    uint8_t maxs[64];            // per region: max s_r (0: no row)
+    uint8_t base[64];            // per region: first row entry
+};
+
+// log2 upper bound of one pattern's fc sum on this diagram:
+// max over programs of sum_t k_t log2(Z[A_t] + 1), Z[A] = vertices covering A
+// (prod_t C(Z_t, k_t) bounds each program's fc); the caller adds T.slack
+__device__ __noinline__ float venn_bound_log2(const uint32_t* venn, int q, const CoreProg& P) {
+    const int V = 1 << q;
+    uint32_t Z[64];
+    for (int A = 0; A < V; ++A) Z[A] = A ? venn[A] : 0;
+    for (int bb = 0; bb < q; ++bb)
+        for (int A = 0; A < V; ++A)
+            if (!(A >> bb & 1)) Z[A] += Z[A | (1 << bb)];
+    float mx = 0.f;
+    for (int pi = 0; pi < P.nprog; ++pi) {
+        const FringeProg& fp = P.prog[pi];
+        float b = 0.f;
+        for (int t = 0; t < fp.s; ++t) b += (float)fp.k[t] * log2f((float)Z[fp.anch[t]] + 1.f);
+        mx = fmaxf(mx, b);
+    }
+    return mx;
+}
+
+// one diagram, every term of the pass, arithmetic mod 2^bits(W): exact when
+// each pattern's fc sum (>= every term, every partial sum) is below
+// 2^(bits - 9): then every used row entry C(n, s) and s * C(n, s) fit too
+template <class W, int NP>
+__device__ __forceinline__ void venn_terms_eval(const uint32_t* venn, int V, const VennDev& T, W* R, int stride,
+                                                AccN<NP>& acc) {
+    for (int r = 1; r < V; ++r) {      // R[base[r] + j - 1] = C(n_r, j), j = 1..maxs[r]
+        const int K = T.maxs[r];
+        if (!K) continue;
+        const uint64_t n = venn[r];
+        W* Rr = R + T.base[r] * stride;
+        W c = 1;
+        for (int j = 1; j <= K; ++j) {
+            c = ((c * (W)(n - (uint64_t)j + 1)) >> c_tz[j]) * inv_odd(j, c);
+            Rr[(j - 1) * stride] = c;
+        }
+    }
+    W sum = 0;
+    int cur = T.terms[0].pat;
+    for (int t = 0; t < T.n; ++t) {
+        const VTerm* e = T.terms + t;
+        const uint64_t cf = __ldg(&e->coef);
+        const uint2 hd = __ldg(reinterpret_cast<const uint2*>(e) + 1);
+        const uint2 tl = __ldg(reinterpret_cast<const uint2*>(e) + 2);
+        const int pat = hd.x & 255, nz = (hd.x >> 8) & 255;
+        if (pat != cur) { acc.add(cur, (u128)sum, false); sum = 0; cur = pat; }
+        // off[0..1] in hd.x bits 16..31, off[2..5] in hd.y, off[6..13] in tl
+        W pr = (W)cf;
+        const uint32_t words[4] = {hd.x >> 16, hd.y, tl.x, tl.y};
+#pragma unroll
+        for (int i = 0; i < kMaxVennNz; ++i) {   // constant shifts, no local memory
+            if (i >= nz) break;
+            const int o = i < 2 ? (int)((words[0] >> (8 * i)) & 255)
+                                : (int)((words[1 + (i - 2) / 4] >> (8 * ((i - 2) & 3))) & 255);
+            pr *= R[o * stride];
+        }
+        sum += pr;
+    }
+    acc.add(cur, (u128)sum, false);
+}
+
+// ------------------------------------------------------------------------
 // Triangle cores (p = 3, all pairs adjacent; symmetry broken u < v < w).
 //
 // Enumeration: one lane per oriented root edge (u, v), merging the short
@@ -738,7 +834,9 @@ constexpr int kTriStack = 32;
 template <int NP>
 __global__ void __launch_bounds__(kTriWarps * 32) tri_core_kernel(GraphDev G, OrientDev O, HubDev H,
                                                                    const CoreProg P, WorkDesc W,
-                                                                   const int* __restrict__ sup, const Sink S) {
+                                                                   const int* __restrict__ sup, const VennDev VD,
+                                                                   const Sink S) {
+    extern __shared__ u128 s_rows[];                 // Venn-table binomial rows [entry][thread]
     __shared__ uint32_t s_leaf[kTriWarps][64][6];   // u, v, w, e(uv), e(uw), e(vw)
     __shared__ uint32_t s_venn[kTriWarps][64][8];   // Venn over the q anchors
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
@@ -833,16 +931,43 @@ __global__ void __launch_bounds__(kTriWarps * 32) tri_core_kernel(GraphDev G, Or
             }
         }
         __syncwarp();
-        // (2) fc over (leaf, program) pairs
-        const int pairs = cnt * nprog;
-        for (int tpair = lane; tpair < pairs; tpair += 32) {
-            const int li = tpair / nprog, pi = tpair - li * nprog;
-            uint32_t vloc[8];
-            for (int k = 0; k < V; ++k) vloc[k] = s_venn[wib][li][k];
-            const FringeProg fp = P.prog[pi];
-            bool o = false;
-            const u128 f = fc_dispatch<kTriStack>(vloc, q, fp, o);
-            acc.add(fp.pat, f, o);
+        if (VD.n) {
+            // (2) fc by the Venn term table, one leaf per lane, every program
+            for (int base = 0; base < cnt; base += 32) {
+                const int li = base + lane;
+                const bool mine = li < cnt;
+                uint32_t vloc[8];
+                float bnd = 0.f;
+                if (mine) {
+                    for (int k = 0; k < V; ++k) vloc[k] = s_venn[wib][li][k];
+                    bnd = venn_bound_log2(vloc, q, P) + VD.slack;
+                }
+                const bool all64 = __all_sync(FULLMASK, !mine || bnd < 55.f);
+                if (mine && all64) {
+                    venn_terms_eval<uint64_t>(vloc, V, VD, (uint64_t*)s_rows + threadIdx.x, blockDim.x, acc);
+                } else if (mine && bnd < 119.f) {
+                    venn_terms_eval<u128>(vloc, V, VD, s_rows + threadIdx.x, blockDim.x, acc);
+                } else if (mine) {                     // checked Listing 5 per program
+                    for (int pi = 0; pi < nprog; ++pi) {
+                        const FringeProg fp = P.prog[pi];
+                        bool o = false;
+                        const u128 f = fc_dispatch<kTriStack>(vloc, q, fp, o);
+                        acc.add(fp.pat, f, o);
+                    }
+                }
+            }
+        } else {
+            // (2) fc over (leaf, program) pairs
+            const int pairs = cnt * nprog;
+            for (int tpair = lane; tpair < pairs; tpair += 32) {
+                const int li = tpair / nprog, pi = tpair - li * nprog;
+                uint32_t vloc[8];
+                for (int k = 0; k < V; ++k) vloc[k] = s_venn[wib][li][k];
+                const FringeProg fp = P.prog[pi];
+                bool o = false;
+                const u128 f = fc_dispatch<kTriStack>(vloc, q, fp, o);
+                acc.add(fp.pat, f, o);
+            }
         }
         nmatch += (lane == 0) ? (unsigned long long)cnt : 0ull;
         cnt = 0;
@@ -981,7 +1106,8 @@ template <int NP>
 __global__ void __launch_bounds__(kCoreWarps * 32) core_kernel(GraphDev G, OrientDev O, HubDev H,
                                                                 const CoreProg P, WorkDesc W,
                                                                 const int* __restrict__ sup, TermDev TD,
-                                                                const Sink S, unsigned long long* queue) {
+                                                                const VennDev VD, const Sink S,
+                                                                unsigned long long* queue) {
     extern __shared__ uint32_t smem[];
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     const int q = P.q, V = 1 << q, p = P.p, nprog = P.nprog;
@@ -1137,7 +1263,30 @@ __global__ void __launch_bounds__(kCoreWarps * 32) core_kernel(GraphDev G, Orien
             __syncwarp();
         }
         __syncwarp();
-        const int pairs = cnt * nprog;            // fc over (leaf, program) pairs
+        if (VD.n) {                               // fc by the Venn term table, leaf per lane
+            u128* rows = reinterpret_cast<u128*>(smem + kCoreWarps * 32 * (FSGC_MAXC + V));
+            const bool mine = lane < cnt;
+            uint32_t vloc[1 << FSGC_MAXQ];
+            float bnd = 0.f;
+            if (mine) {
+                for (int k = 0; k < V; ++k) vloc[k] = s_venn[lane * V + k];
+                bnd = venn_bound_log2(vloc, q, P) + VD.slack;
+            }
+            const bool all64 = __all_sync(FULLMASK, !mine || bnd < 55.f);
+            if (mine && all64) {
+                venn_terms_eval<uint64_t>(vloc, V, VD, (uint64_t*)rows + threadIdx.x, blockDim.x, acc);
+            } else if (mine && bnd < 119.f) {
+                venn_terms_eval<u128>(vloc, V, VD, rows + threadIdx.x, blockDim.x, acc);
+            } else if (mine) {
+                for (int pi = 0; pi < nprog; ++pi) {
+                    bool o = false;
+                    const FringeProg fp = P.prog[pi];
+                    const u128 f = fc_dispatch<FSGC_FC_STACK>(vloc, q, fp, o);
+                    acc.add(fp.pat, f, o);
+                }
+            }
+        }
+        const int pairs = VD.n ? 0 : cnt * nprog;  // else fc over (leaf, program) pairs
         for (int tp = lane; tp < pairs; tp += 32) {
             const int l2 = tp / nprog, pi = tp - l2 * nprog;
             uint32_t vloc[1 << FSGC_MAXQ];
@@ -1436,14 +1585,17 @@ struct PassExec {
     PassPlan plan;
     int kind = 0;              // 0 vertex, 1 edge (support + fc), 2 general core
     int npc = 1;               // accumulator width class
-    int64_t grid = 1, grid_sup = 1;
+    int64_t grid = 1;
     size_t smem = 0;
     WorkDesc W{};
-    size_t ws_off = 0, sup_bytes = 0, parts_off = 0, bytes = 0;
+    bool uses_sup = false;     // reads the plan's per-edge support array
+    size_t ws_off = 0, parts_off = 0, bytes = 0;
     int term_base = 0;         // index of this pass's programs in the term offset/count arrays
     bool whole = true;
     EdgeTerms et{};            // edge cores: the Sec. 3.1 term table (et.n == 0: checked path)
     size_t smem_fc = 0;        // dynamic shared memory of edge_fc_kernel
+    VennDev vd{};              // triangle / general cores: the Venn term table (vd.n == 0: off)
+    size_t smem_vd = 0;        // its per-thread binomial rows (dynamic shared memory)
 };
 
 // the term table of an edge-core pass (see EdgeTerms); et.n = 0 when a
@@ -1481,6 +1633,89 @@ static void build_edge_terms(const CoreProg& cp, EdgeTerms* et) {
     et->ka = ka; et->kb = kb; et->kc = kc;
     et->kmax = kmax;
 }
+
+// the Venn term table of a triangle / general-core pass (see VTerm): walk
+// Listing 5's tree of every program on the host -- type by type, the next
+// covering region with x > 0 fringes, s_r += x, coef *= C(s_r, x) (the
+// multinomial split of region r built up one type at a time) -- and merge
+// the leaves by (pattern, s).  Returns false (table off: per-program
+// Listing 5 on the device) past the size limits or a 64-bit coefficient.
+static bool build_venn_terms(const CoreProg& cp, std::vector<VTerm>* out, VennDev* hd) {
+    const int q = cp.q, V = 1 << q;
+    std::memset(hd, 0, sizeof *hd);
+    out->clear();
+    std::map<std::pair<int, std::vector<uint8_t>>, u128> acc;
+    long long leaves = 0;
+    const long long kLeafCap = 4000000;
+    bool ok = true;
+    int progs_per_pat[FSGC_MAXPATS] = {0};
+    for (int pi = 0; pi < cp.nprog && ok; ++pi) {
+        const FringeProg& fp = cp.prog[pi];
+        ++progs_per_pat[fp.pat];
+        std::vector<uint8_t> sv(V, 0);
+        std::function<void(int, int, int, u128)> rec = [&](int t, int r0, int rem, u128 coef) {
+            if (!ok) return;
+            if (rem == 0) {
+                if (t + 1 == fp.s || fp.s == 0) {
+                    if (++leaves > kLeafCap) { ok = false; return; }
+                    bool o = false;
+                    u128& a = acc[std::make_pair((int)fp.pat, sv)];
+                    a = add_ovf(a, coef, o);
+                    if (o) ok = false;
+                    return;
+                }
+                rec(t + 1, 1, fp.k[t + 1], coef);
+                return;
+            }
+            const int A = fp.anch[t];
+            for (int r = r0; r < V; ++r) {
+                if ((r & A) != A) continue;
+                for (int x = 1; x <= rem; ++x) {
+                    sv[r] += (uint8_t)x;
+                    bool o = false;
+                    const u128 c = mul_ovf(coef, binom_ovf(sv[r], (uint32_t)x, o), o);
+                    if (o) ok = false;
+                    else rec(t, r + 1, rem - x, c);
+                    sv[r] -= (uint8_t)x;
+                }
+            }
+        };
+        if (fp.s == 0) rec(0, 1, 0, 1);
+        else rec(0, 1, fp.k[0], 1);
+    }
+    if (!ok || acc.empty() || (int)acc.size() > kMaxVennTerms) return false;
+    int maxs[64] = {0};
+    for (auto& kv : acc) {
+        if (kv.second >> 64) return false;
+        int nz = 0;
+        for (int r = 1; r < V; ++r)
+            if (kv.first.second[r]) { ++nz; maxs[r] = std::max(maxs[r], (int)kv.first.second[r]); }
+        if (nz > kMaxVennNz) return false;
+    }
+    int nrows = 0;
+    for (int r = 1; r < V; ++r) {
+        if (maxs[r] > 63) return false;
+        hd->maxs[r] = (uint8_t)maxs[r];
+        hd->base[r] = (uint8_t)nrows;
+        nrows += maxs[r];
+    }
+    if (nrows > kMaxVennRows) return false;
+    for (auto& kv : acc) {
+        VTerm t;
+        std::memset(&t, 0, sizeof t);
+        t.coef = (uint64_t)kv.second;
+        t.pat = (uint8_t)kv.first.first;
+        for (int r = 1; r < V; ++r)
+            if (kv.first.second[r]) t.off[t.nz++] = (uint8_t)(hd->base[r] + kv.first.second[r] - 1);
+        out->push_back(t);
+    }
+    int mp = 1;
+    for (int i = 0; i < FSGC_MAXPATS; ++i) mp = std::max(mp, progs_per_pat[i]);
+    hd->n = (int32_t)out->size();
+    hd->nrows = nrows;
+    hd->slack = std::log2((float)mp) + 2.f;
+    return true;
+}
 }  // namespace
 
 // device copies of the partition-lattice term tables of a pattern batch;
@@ -1490,10 +1725,13 @@ struct DevTerms {
     PartTerm* terms = nullptr;
     int32_t* off = nullptr;
     int32_t* cnt = nullptr;
+    VTerm* vterms = nullptr;        // Venn term tables of all passes
+    std::vector<VennDev> vhdr;      // per pass (terms point into vterms)
     ~DevTerms() {
         if (terms) cudaFree(terms);
         if (off) cudaFree(off);
         if (cnt) cudaFree(cnt);
+        if (vterms) cudaFree(vterms);
     }
 };
 
@@ -1504,7 +1742,13 @@ struct fsgc_plan {
     size_t ws_bytes = 0;
     int publish_mode = 1;
     int device = 0;
-    std::vector<cudaEvent_t> ev;   // 3 per pass
+    // one per-edge support array c(e) = |N(u) & N(v)| for every pass that
+    // reads it (edge, triangle and general cores), at ws[sup_off, + 4 m)
+    int sup_first = -1;            // first pass reading it (-1: none)
+    size_t sup_off = 0;
+    int64_t grid_sup = 1;
+    int sup_shard = 0, sup_nshards = 1;   // FSGC_FLAG_SHARD_SUPPORT: this shard's part
+    std::vector<cudaEvent_t> ev;   // support begin/end, then begin/end per pass
     unsigned long long* trace = nullptr;
     std::shared_ptr<DevTerms> terms;   // partition-lattice terms of all programs
     ~fsgc_plan() {
@@ -1565,8 +1809,6 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
             X.grid = std::max<int64_t>(1, std::min<int64_t>((work + 255) / 256,
                                                             (int64_t)nsm * occupancy(kernel_for(0, X.npc), 256, 0)));
         } else if (X.kind == 1) {
-            X.grid_sup = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy((const void*)support_kernel, 256, 0),
-                                                                (g->m + 255) / 256));
             int64_t mine = ((e - b) + 31) / 32;
             mine = (mine + opts.shard_count - 1) / opts.shard_count;
             build_edge_terms(cp, &X.et);
@@ -1575,28 +1817,35 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
             X.grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy(kernel_for(1, X.npc), 256, X.smem_fc),
                                                             (mine + 7) / 8));
             if (tune("FSGC_EDGE_BLOCKS", 0) > 0) X.grid = tune("FSGC_EDGE_BLOCKS", 0);
-            X.sup_bytes = (size_t)std::max<int64_t>(g->m, 1) * sizeof(int);
         } else if (X.kind == 3) {
-            X.grid_sup = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy((const void*)support_kernel, 256, 0),
-                                                                (g->m + 255) / 256));
             int64_t mine = ((e - b) + 31) / 32;
             mine = (mine + opts.shard_count - 1) / opts.shard_count;
             X.grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy(kernel_for(3, X.npc), kTriWarps * 32, 0),
                                                             (mine + kTriWarps - 1) / kTriWarps));
-            X.sup_bytes = (size_t)std::max<int64_t>(g->m, 1) * sizeof(int);
         } else {
             X.smem = (size_t)kCoreWarps * (32 * FSGC_MAXC + 32 * (1u << cp.q)) * sizeof(uint32_t);
             int64_t nchunks = ((e - b) + X.W.chunk - 1) / X.W.chunk;
             int64_t mine = (nchunks + opts.shard_count - 1) / opts.shard_count;
             X.grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy(kernel_for(2, X.npc), kCoreWarps * 32, X.smem),
                                                             (mine + kCoreWarps - 1) / kCoreWarps));
-            X.sup_bytes = (size_t)std::max<int64_t>(g->m, 1) * sizeof(int);
         }
-        X.parts_off = (kHdrBytes + X.sup_bytes + 255) & ~(size_t)255;
+        X.uses_sup = X.kind != 0 && g->m > 0;
+        if (X.uses_sup && P->sup_first < 0) P->sup_first = (int)P->passes.size();
+        X.parts_off = kHdrBytes;
         X.bytes = (X.parts_off + (size_t)X.grid * sizeof(BlockPartial) + 255) & ~(size_t)255;
         X.ws_off = off;
         off += X.bytes;
         P->passes.push_back(X);
+    }
+    if (P->sup_first >= 0) {
+        P->sup_off = off;
+        off += ((size_t)g->m * sizeof(int) + 255) & ~(size_t)255;
+        P->grid_sup = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy((const void*)support_kernel, 256, 0),
+                                                             (g->m + 255) / 256));
+        if ((opts.flags & FSGC_FLAG_SHARD_SUPPORT) && opts.shard_count > 1) {
+            P->sup_shard = opts.shard_index;
+            P->sup_nshards = opts.shard_count;
+        }
     }
     P->ws_bytes = off;
     {   // partition-lattice term tables -> device (cached)
@@ -1629,12 +1878,47 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
             FSGC_CUDA(cudaMemcpy(T->terms, all.data(), all.size() * sizeof(PartTerm), cudaMemcpyHostToDevice));
             FSGC_CUDA(cudaMemcpy(T->off, offs.data(), offs.size() * sizeof(int32_t), cudaMemcpyHostToDevice));
             FSGC_CUDA(cudaMemcpy(T->cnt, cnts.data(), cnts.size() * sizeof(int32_t), cudaMemcpyHostToDevice));
+            // Venn term tables (pattern-only, so cached with the rest)
+            std::vector<VTerm> vall;
+            std::vector<size_t> vbase;
+            for (auto& X : P->passes) {
+                VennDev hd;
+                std::memset(&hd, 0, sizeof hd);
+                std::vector<VTerm> vt;
+                if ((X.kind == 2 || X.kind == 3) && !tune("FSGC_NO_VENN_TERMS", 0) &&
+                    build_venn_terms(X.plan.prog, &vt, &hd)) {
+                    vbase.push_back(vall.size());
+                    vall.insert(vall.end(), vt.begin(), vt.end());
+                } else {
+                    std::memset(&hd, 0, sizeof hd);
+                    vbase.push_back(0);
+                }
+                T->vhdr.push_back(hd);
+            }
+            if (!vall.empty()) {
+                FSGC_CUDA(cudaMalloc(&T->vterms, vall.size() * sizeof(VTerm)));
+                FSGC_CUDA(cudaMemcpy(T->vterms, vall.data(), vall.size() * sizeof(VTerm), cudaMemcpyHostToDevice));
+            }
+            for (size_t i = 0; i < T->vhdr.size(); ++i)
+                if (T->vhdr[i].n) T->vhdr[i].terms = T->vterms + vbase[i];
             if (tcache.size() > 256) tcache.clear();
             tcache[tkey] = T;
             P->terms = T;
         }
+        // Venn tables -> passes: rows in dynamic shared memory, grids re-sized
+        const size_t kStatic = 40 * 1024;    // the kernels' static shared memory (upper bound)
+        for (size_t i = 0; i < P->passes.size(); ++i) {
+            PassExec& X = P->passes[i];
+            X.vd = P->terms->vhdr[i];
+            if (!X.vd.n) continue;
+            const int threads = X.kind == 3 ? kTriWarps * 32 : kCoreWarps * 32;
+            X.smem_vd = (size_t)X.vd.nrows * sizeof(u128) * threads;
+            if (X.smem_vd + X.smem + kStatic > 227 * 1024) { X.vd.n = 0; X.smem_vd = 0; continue; }
+            const int64_t per = (int64_t)nsm * occupancy(kernel_for(X.kind, X.npc), threads, X.smem + X.smem_vd);
+            X.grid = std::max<int64_t>(1, std::min<int64_t>(X.grid, per));
+        }
     }
-    P->ev.resize(3 * P->passes.size());
+    P->ev.resize(2 + 2 * P->passes.size());
     for (auto& ev : P->ev) FSGC_CUDA(cudaEventCreate(&ev));
     if (tune("FSGC_TRACE", 0)) {
         FSGC_CUDA(cudaMalloc(&P->trace, (size_t)2 * 1024 * 1024));
@@ -1651,8 +1935,17 @@ extern "C" int fsgc_plan_workspace_bytes(const fsgc_plan* P, size_t* ws, size_t*
     return FSGC_OK;
 }
 
-extern "C" int fsgc_plan_enqueue(const fsgc_plan* P, void* workspace, void* raw_out, void* stream_) {
+extern "C" int fsgc_plan_support_region(const fsgc_plan* P, size_t* offset, int64_t* count) {
+    if (!P || !offset || !count) FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_plan_support_region: null argument");
+    *offset = P->sup_off;
+    *count = P->sup_first >= 0 ? P->g->m : 0;
+    return FSGC_OK;
+}
+
+extern "C" int fsgc_plan_enqueue_stage(const fsgc_plan* P, void* workspace, void* raw_out, int stages,
+                                       void* stream_) {
     if (!P || !workspace || !raw_out) FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_plan_enqueue: null argument");
+    if (stages & ~FSGC_STAGE_ALL) FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_plan_enqueue_stage: bad stage mask %d", stages);
     cudaStream_t st = (cudaStream_t)stream_;
     cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
     FSGC_CUDA(cudaStreamIsCapturing(st, &cap));
@@ -1661,25 +1954,29 @@ extern "C" int fsgc_plan_enqueue(const fsgc_plan* P, void* workspace, void* raw_
     const fsgc_graph* g = P->g;
     GraphDev G{g->offsets, g->adj, g->row, g->osrc, g->odst};
     OrientDev O{g->split, g->oofs};
+    int* dsup = (int*)((unsigned char*)workspace + P->sup_off);
+    if ((stages & FSGC_STAGE_SUPPORT) && P->sup_first >= 0) {   // (A) per-edge common-neighbour counts
+        FSGC_CUDA(cudaMemsetAsync(dsup, 0, (size_t)g->m * sizeof(int), st));
+        FSGC_CUDA(cudaEventRecordWithFlags(P->ev[0], st, evflags));
+        support_kernel<<<(int)P->grid_sup, 256, 0, st>>>(G, O, g->m, dsup, g->sorder, g->ssrc, g->sdst,
+                                                          P->sup_shard, P->sup_nshards,
+                                                          P->trace ? P->trace + (1 << 17) : nullptr);
+        FSGC_CUDA(cudaGetLastError());
+        FSGC_CUDA(cudaEventRecordWithFlags(P->ev[1], st, evflags));
+    }
+    if (!(stages & FSGC_STAGE_COUNT)) return FSGC_OK;
     for (size_t pi = 0; pi < P->passes.size(); ++pi) {
         const PassExec& X = P->passes[pi];
         unsigned char* base = (unsigned char*)workspace + X.ws_off;
-        FSGC_CUDA(cudaMemsetAsync(base, 0, kHdrBytes + X.sup_bytes, st));
+        FSGC_CUDA(cudaMemsetAsync(base, 0, kHdrBytes, st));
         AccDev* dacc = (AccDev*)base;
         unsigned long long* dmatch = (unsigned long long*)(base + sizeof(AccDev) * FSGC_MAXPATS);
         unsigned long long* dqueue = dmatch + 1;
         unsigned int* dticket = (unsigned int*)(dmatch + 3);
-        int* dsup = (int*)(base + kHdrBytes);
         Sink S{dacc, dmatch, (BlockPartial*)(base + X.parts_off), dticket, P->publish_mode};
         WorkDesc W = X.W;
         const CoreProg& cp = X.plan.prog;
-        FSGC_CUDA(cudaEventRecordWithFlags(P->ev[3 * pi], st, evflags));
-        if (X.kind != 0 && g->m > 0) {   // (A) per-edge common-neighbour counts
-            support_kernel<<<(int)X.grid_sup, 256, 0, st>>>(G, O, g->m, dsup, g->sorder, g->ssrc, g->sdst,
-                                                             P->trace ? P->trace + (1 << 17) : nullptr);
-            FSGC_CUDA(cudaGetLastError());
-        }
-        FSGC_CUDA(cudaEventRecordWithFlags(P->ev[3 * pi + 1], st, evflags));
+        FSGC_CUDA(cudaEventRecordWithFlags(P->ev[2 + 2 * pi], st, evflags));
         if (W.end > W.begin) {
             const void* fn = kernel_for(X.kind, X.npc);
             void* args_v[] = {(void*)&G, (void*)&cp, (void*)&W, (void*)&S};
@@ -1687,22 +1984,31 @@ extern "C" int fsgc_plan_enqueue(const fsgc_plan* P, void* workspace, void* raw_
             HubDev Hd{g->hub_base, g->hub_words, g->hub_bits};
             TermDev TD{P->terms->terms, P->terms->off + X.term_base, P->terms->cnt + X.term_base};
             void* args_c[] = {(void*)&G, (void*)&O, (void*)&Hd, (void*)&cp, (void*)&W, (void*)&dsup, (void*)&TD,
-                              (void*)&S, (void*)&dqueue};
-            void* args_t[] = {(void*)&G, (void*)&O, (void*)&Hd, (void*)&cp, (void*)&W, (void*)&dsup, (void*)&S};
+                              (void*)&X.vd, (void*)&S, (void*)&dqueue};
+            void* args_t[] = {(void*)&G, (void*)&O, (void*)&Hd, (void*)&cp, (void*)&W, (void*)&dsup, (void*)&X.vd,
+                              (void*)&S};
             if (X.kind == 0)
                 FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(256), args_v, 0, st));
             else if (X.kind == 1)    // (B) fringe counts per root edge
                 FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(256), args_e, X.smem_fc, st));
             else if (X.kind == 3)
-                FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(kTriWarps * 32), args_t, 0, st));
+                FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(kTriWarps * 32), args_t, X.smem_vd, st));
             else
-                FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(kCoreWarps * 32), args_c, X.smem, st));
+                FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(kCoreWarps * 32), args_c,
+                                           X.smem + X.smem_vd, st));
         }
-        FSGC_CUDA(cudaEventRecordWithFlags(P->ev[3 * pi + 2], st, evflags));
+        FSGC_CUDA(cudaEventRecordWithFlags(P->ev[3 + 2 * pi], st, evflags));
         FSGC_CUDA(cudaMemcpyAsync((unsigned char*)raw_out + pi * kRawPassBytes, base, kRawPassBytes - 8,
                                   cudaMemcpyDefault, st));
     }
     return FSGC_OK;
+}
+
+extern "C" int fsgc_plan_enqueue(const fsgc_plan* P, void* workspace, void* raw_out, void* stream_) {
+    if (P && P->sup_nshards > 1)
+        FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_plan_enqueue: a plan with a sharded support pass runs in two "
+                                    "stages (fsgc_plan_enqueue_stage) with the support sum in between");
+    return fsgc_plan_enqueue_stage(P, workspace, raw_out, FSGC_STAGE_ALL, stream_);
 }
 
 extern "C" int fsgc_plan_decode(const fsgc_plan* P, const void* raw, fsgc_result* results) {
@@ -1713,11 +2019,13 @@ extern "C" int fsgc_plan_decode(const fsgc_plan* P, const void* raw, fsgc_result
         const AccDev* acc = (const AccDev*)((const unsigned char*)raw + pi * kRawPassBytes);
         unsigned long long matches;
         std::memcpy(&matches, (const unsigned char*)raw + pi * kRawPassBytes + sizeof(AccDev) * FSGC_MAXPATS, 8);
+        // the shared support pass is reported with the first pass reading it
+        const bool sup_here = (int)pi == P->sup_first;
         float kms = 0.f, ams = 0.f;
-        if (cudaEventElapsedTime(&ams, P->ev[3 * pi], P->ev[3 * pi + 1]) != cudaSuccess) ams = -1.f;
-        if (cudaEventElapsedTime(&kms, P->ev[3 * pi + 1], P->ev[3 * pi + 2]) != cudaSuccess) kms = -1.f;
+        if (sup_here && cudaEventElapsedTime(&ams, P->ev[0], P->ev[1]) != cudaSuccess) ams = -1.f;
+        if (cudaEventElapsedTime(&kms, P->ev[2 + 2 * pi], P->ev[3 + 2 * pi]) != cudaSuccess) kms = -1.f;
         cudaGetLastError();   // timing is best effort (e.g. events recorded inside a graph)
-        const int launches = (X.W.end > X.W.begin ? 1 : 0) + (X.kind != 0 && P->g->m > 0 ? 1 : 0);
+        const int launches = (X.W.end > X.W.begin ? 1 : 0) + (sup_here ? 1 : 0);
         for (size_t mi = 0; mi < X.plan.members.size(); ++mi) {
             fsgc_result& r = results[X.plan.members[mi]];
             r.raw.lo = acc[mi].lo;
@@ -1837,6 +2145,9 @@ extern "C" int fsgc_count(const fsgc_graph* g, const fsgc_pattern* const* pats, 
         FSGC_CUDA(cudaMallocHost(&tb.raw, std::max<size_t>(rawb, 4096)));
         tb.raw_size = std::max<size_t>(rawb, 4096);
     }
+    if (plan->sup_nshards > 1)
+        FSGC_FAIL(FSGC_ERR_INVALID, "fsgc_count: FSGC_FLAG_SHARD_SUPPORT needs the staged plan API "
+                                    "(the shards' support arrays are summed between the stages)");
     int rc = fsgc_plan_enqueue(plan.get(), tb.ws, tb.raw, st);
     if (rc) return rc;
     FSGC_CUDA(cudaStreamSynchronize(st));

@@ -15,6 +15,8 @@
 // osrc/odst int32[m] (SoA, sorted by (u, v)), order int32[n].
 #include <cub/cub.cuh>
 #include <atomic>
+#include <mutex>
+#include <set>
 #include <cstdlib>
 #include <vector>
 #include <algorithm>
@@ -193,6 +195,23 @@ int grid_for(int64_t work) {
     return (int)g;
 }
 
+// The build's temporaries come from the device's default stream-ordered pool.
+// With its default release threshold (0) every synchronisation hands the freed
+// pages back to the driver and the next load maps them again; keep up to
+// 8 GiB cached instead (once per device).
+cudaError_t keep_pool_memory(int dev) {
+    static std::mutex mu;
+    static std::set<int> done;
+    std::lock_guard<std::mutex> lock(mu);
+    if (done.count(dev)) return cudaSuccess;
+    cudaMemPool_t pool;
+    cudaError_t e = cudaDeviceGetDefaultMemPool(&pool, dev);
+    if (e != cudaSuccess) return e;
+    uint64_t keep = 8ull << 30;
+    e = cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+    if (e == cudaSuccess) done.insert(dev);
+    return e;
+}
 }  // namespace
 
 extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, int on_device,
@@ -205,6 +224,7 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
     cudaStream_t st = (cudaStream_t)stream_;
     int dev = 0;
     FSGC_CUDA(cudaGetDevice(&dev));
+    FSGC_CUDA(keep_pool_memory(dev));
 
     int B = 1;
     while ((1ll << B) < n) ++B;

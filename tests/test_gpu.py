@@ -309,3 +309,114 @@ def test_edge_core_counts_beyond_64_bits():
     assert any(r.count is not None and r.count >= 1 << 64 for r in res)
     for P, r in zip(pats, res):
         assert not r.overflow and r.count == oracle.fringe_count(gadj, P.n, P.edges, P.core), P.name
+
+
+def test_sharded_support_stages_sum_to_whole():
+    """FSGC_FLAG_SHARD_SUPPORT: each shard lists its interleaved part of the
+    triangles into a partial support array; the SUM of the partial arrays
+    (what the multi-GPU all-reduce computes) is the full support array, and
+    stage 2 on it gives per-shard raws that sum to the unsharded raw -- for
+    an edge-core, a triangle-core and a general-core pass in one plan."""
+    from paper_conf_sc_bradleyab25_b200 import _lib
+    n, e, _ = workload("pl2k")
+    g = F.fsgc_load_graph(e, n)
+    pats = [F.compile_named(PATTERNS[x]) for x in ["2-tailed-triangle", "tricore+3f", "k4core+2f", "cycle4"]]
+    whole = F.fsgc_count(g, pats)
+    full = F.Plan(g, pats)
+    full.enqueue()
+    torch.cuda.synchronize()
+    ref_sup = full.support().clone()
+    assert int(ref_sup.sum()) > 0
+    for shards in (2, 3):
+        plans = [F.Plan(g, pats, shard_index=s, shard_count=shards, shard_support=True) for s in range(shards)]
+        for P in plans:
+            P.enqueue_stage(_lib.FSGC_STAGE_SUPPORT)
+        torch.cuda.synchronize()
+        tot = sum(P.support().to(torch.int64) for P in plans)
+        assert torch.equal(tot.to(torch.int32), ref_sup)
+        for P in plans:
+            assert not torch.equal(P.support(), ref_sup)      # each part really is partial
+            P.support().copy_(tot.to(torch.int32))
+            P.enqueue_stage(_lib.FSGC_STAGE_COUNT)
+        torch.cuda.synchronize()
+        raws = [0] * len(pats)
+        for P in plans:
+            for k, r in enumerate(P.decode()):
+                raws[k] += r.raw
+        assert raws == [r.raw for r in whole]
+    with pytest.raises(F.FsgcError):
+        F.fsgc_count(g, pats, shard_index=0, shard_count=2, shard_support=True)
+    with pytest.raises(F.FsgcError):
+        F.Plan(g, pats, shard_index=0, shard_count=2, shard_support=True).enqueue()
+
+
+def _dist_worker(rank, world, port, q):
+    import os
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    import torch.distributed as dist
+    torch.cuda.set_device(0)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    n, e = workload_edges("pl2k")
+    g = F.fsgc_load_graph(e, n)
+    names = ["1-tailed-triangle", "tricore+2f", "diamond", "3-star"]
+    pats = [F.compile_named(PATTERNS[x]) for x in names]
+    res = F.fsgc_count_distributed(g, pats)
+    if rank == 0:
+        q.put([r.count for r in res])
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_count_distributed_two_ranks_gloo_on_one_gpu():
+    """fsgc_count_distributed end to end with 2 ranks (gloo over CUDA tensors,
+    both on cuda:0): sharded support + all-reduce, sharded roots + the
+    128-bit all-reduce == the single-process count."""
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = 29500 + random.Random().randint(0, 2000)
+    procs = [ctx.Process(target=_dist_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    got = q.get(timeout=300)
+    for p in procs:
+        p.join(timeout=120)
+        assert p.exitcode == 0
+    n, e, _ = workload("pl2k")
+    g = F.fsgc_load_graph(e, n)
+    names = ["1-tailed-triangle", "tricore+2f", "diamond", "3-star"]
+    want = [r.count for r in F.fsgc_count(g, [F.compile_named(PATTERNS[x]) for x in names])]
+    assert got == want
+
+
+def test_venn_term_table_tiers_vs_oracle():
+    """Triangle- and 4-clique-core counts through the Venn term table in all
+    three arithmetic tiers -- 64-bit (small leaf triangles), 128-bit and the
+    checked Listing 5 fallback (the hub triangle: 13 fringes over ~2^11-sized
+    regions, bound > 2^119) -- vs the oracle."""
+    rng = np.random.default_rng(11)
+    A, B, Cc = 0, 1, 2
+    e = [(A, B), (A, Cc), (B, Cc)]
+    nxt = 3
+    for h in (A, B, Cc):
+        for _ in range(3000):
+            e.append((h, nxt)); nxt += 1
+    for _ in range(60):
+        e += [(A, nxt), (B, nxt), (Cc, nxt)]; nxt += 1
+    for x, y in ((A, B), (A, Cc), (B, Cc)):
+        for _ in range(60):
+            e += [(x, nxt), (y, nxt)]; nxt += 1
+    leaves = np.arange(3, nxt)
+    for _ in range(4000):                                  # small triangles among the leaves
+        a, b = rng.choice(leaves, 2, replace=False)
+        e.append((int(a), int(b)))
+    n = nxt
+    e = np.array(e, dtype=np.int64)
+    _, _, _, gadj = oracle_graph(n, e)
+    names = ["fig4", "tricore+6f", "clique4", "k4core+6f"]
+    pats = [PATTERNS[x] for x in names]
+    g = F.fsgc_load_graph(e, n)
+    res = F.fsgc_count(g, [F.compile_named(P) for P in pats])
+    assert res[0].count is not None and res[0].count >= 1 << 100
+    for P, r in zip(pats, res):
+        assert not r.overflow and r.count == oracle.fringe_count(gadj, P.n, P.edges, P.core), P.name
