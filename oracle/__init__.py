@@ -32,5 +32,5 @@ from .pattern import (  # noqa: F401
 )
 from .count import (  # noqa: F401
     count_monomorphisms, brute_force_count, fc, venn_sizes, fringe_count,
-    core_matches, root_raw_sum, closed_forms,
+    core_matches, root_raw_sum, closed_forms, k_tailed_triangles,
 )

@@ -587,7 +587,9 @@ __global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, c
             const uint64_t nu = s_q[wib][lane][0], nv = s_q[wib][lane][1], nuv = s_q[wib][lane][2];
             const int nbits = T.n > 0 ? bitlen64(nu + nv + nuv) * T.kmax : 1 << 20;
             if (nbits <= 63) {
-                edge_terms_eval<uint64_t>(nu, nv, nuv, T, (uint64_t*)s_rows + threadIdx.x, stride, acc);
+                // same byte layout as the u128 rows (threads of another tier share the
+                // buffer): entry t of this thread in the low half of its u128 slot
+                edge_terms_eval<uint64_t>(nu, nv, nuv, T, (uint64_t*)(s_rows + threadIdx.x), 2 * stride, acc);
             } else if (nbits <= 127) {
                 edge_terms_eval<u128>(nu, nv, nuv, T, (u128*)s_rows + threadIdx.x, stride, acc);
             } else {
@@ -944,7 +946,7 @@ __global__ void __launch_bounds__(kTriWarps * 32) tri_core_kernel(GraphDev G, Or
                 }
                 const bool all64 = __all_sync(FULLMASK, !mine || bnd < 55.f);
                 if (mine && all64) {
-                    venn_terms_eval<uint64_t>(vloc, V, VD, (uint64_t*)s_rows + threadIdx.x, blockDim.x, acc);
+                    venn_terms_eval<uint64_t>(vloc, V, VD, (uint64_t*)(s_rows + threadIdx.x), 2 * blockDim.x, acc);
                 } else if (mine && bnd < 119.f) {
                     venn_terms_eval<u128>(vloc, V, VD, s_rows + threadIdx.x, blockDim.x, acc);
                 } else if (mine) {                     // checked Listing 5 per program
@@ -1274,7 +1276,7 @@ __global__ void __launch_bounds__(kCoreWarps * 32) core_kernel(GraphDev G, Orien
             }
             const bool all64 = __all_sync(FULLMASK, !mine || bnd < 55.f);
             if (mine && all64) {
-                venn_terms_eval<uint64_t>(vloc, V, VD, (uint64_t*)rows + threadIdx.x, blockDim.x, acc);
+                venn_terms_eval<uint64_t>(vloc, V, VD, (uint64_t*)(rows + threadIdx.x), 2 * blockDim.x, acc);
             } else if (mine && bnd < 119.f) {
                 venn_terms_eval<u128>(vloc, V, VD, rows + threadIdx.x, blockDim.x, acc);
             } else if (mine) {

@@ -420,3 +420,22 @@ def test_venn_term_table_tiers_vs_oracle():
     assert res[0].count is not None and res[0].count >= 1 << 100
     for P, r in zip(pats, res):
         assert not r.overflow and r.count == oracle.fringe_count(gadj, P.n, P.edges, P.core), P.name
+
+
+def test_k_tailed_triangles_rmat16_closed_form():
+    """RMAT-16 (hubs of degree ~6k next to leaf edges): the edge-core pass runs
+    its 64- and 128-bit term-table tiers side by side in one block; every
+    k-tailed triangle count must equal the closed form sum over triangles of
+    C(deg x - 2, k) (oracle.k_tailed_triangles, pinned), in one batch and
+    alone, and twice (deterministic)."""
+    n, e, (_, _, _, gadj) = workload("rmat16")
+    g = F.fsgc_load_graph(e, n)
+    ks = [1, 4]
+    pats = [F.compile_named(PATTERNS[f"{k}-tailed-triangle"]) for k in range(1, 5)]
+    batch = F.fsgc_count(g, pats)
+    again = F.fsgc_count(g, pats)
+    assert [r.raw for r in batch] == [r.raw for r in again]
+    for k in ks:
+        want = oracle.k_tailed_triangles(gadj, k)
+        assert not batch[k - 1].overflow and batch[k - 1].count == want, k
+        assert F.fsgc_count(g, [pats[k - 1]])[0].count == want, k

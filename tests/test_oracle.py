@@ -81,6 +81,15 @@ def test_closed_forms_random(seed):
             assert oracle.brute_force_count(g, P.n, P.edges) == val, name
     cf = oracle.closed_forms(g)
     assert cf["edge"] == m and cf["3-star"] == expect["3-star"]
+    # k-tailed triangles: explicit triples x C(deg - 2, k), vs the brute-force
+    # mode (k <= 2: <= 5 pattern vertices) and the core/fringe mode
+    for k in range(1, 5):
+        want = sum(comb(int(deg[v]) - 2, k) for t in tris for v in t)
+        assert oracle.k_tailed_triangles(g, k) == want
+        P = PATTERNS[f"{k}-tailed-triangle"]
+        assert oracle.fringe_count(g, P.n, P.edges) == want, k
+        if P.n <= 5:
+            assert oracle.brute_force_count(g, P.n, P.edges) == want, k
 
 
 # ------------------------------------------------------------ exhaustive
