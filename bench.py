@@ -47,7 +47,7 @@ WORKLOAD_DESC = {
                 "124,651 V / 193,620 E (BASELINE configs[1])",
     "pl2k": "tailed triangle on synthetic power-law graph 2,000 V / 10,000 E (configs[0])",
     "rmat22": "triangle, diamond and k-tailed triangles (k=1..4) on RMAT scale 22 (configs[2] graph)",
-    "rmat16": "4-clique cores with 1-6 and diamond cores with 1-2 mixed fringes on RMAT scale 16 "
+    "rmat16": "4-clique cores with 1-6 and a diamond core with 1 mixed fringe on RMAT scale 16 "
               "(configs[2] patterns; Table 1's rmat16.sym scale)",
     "pl10m": "Fig. 4 16-vertex/25-edge pattern on synthetic power-law graph, 10M edges (configs[3])",
     "rmat26": "triangle and 4-cycle cores with fringes on RMAT scale 26 (configs[4])",

@@ -143,7 +143,7 @@ CONFIG_PATTERNS = {
     "pl2k": ["1-tailed-triangle"],
     "internet": [f"{k}-tailed-triangle" for k in range(1, 5)],
     "rmat22": ["triangle", "diamond"] + [f"{k}-tailed-triangle" for k in range(1, 5)],
-    "rmat16": [f"k4core+{f}f" for f in range(1, 7)] + [f"diamondcore+{f}f" for f in range(1, 3)],
+    "rmat16": [f"k4core+{f}f" for f in range(1, 7)] + ["diamondcore+1f"],
     "pl10m": ["fig4"],
     "rmat26": [f"tricore+{f}f" for f in range(1, 7)] + [f"c4core+{f}f" for f in range(1, 7)],
 }
