@@ -264,6 +264,7 @@ def main():
         def step():
             return F.fsgc_count_distributed(g, cps)
         replay = None
+        plan = None
     else:
         # one CUDA graph per step: workspace zeroing, every kernel of every
         # pass, and the copy of the raw 128-bit results into pinned memory
@@ -351,9 +352,25 @@ def main():
     indeg = deg - out
     m = g.m
     share = 1.0 / world
-    # support pass: per oriented edge 8 B (u,v) + 32 B (split/offs of u and v)
-    # + 4 B per out-list entry read by the merge (out(u) + out(v)); all edges
-    sup_bytes = 40.0 * m + 4.0 * float((out * out).sum() + (indeg * out).sum())
+    # support pass: wedge-hash part -- per in-entry
+    # (a, b) of a table middle b: 4 B a + 4 B rev + 24 B split/oofs/offs of a,
+    # 4 B per tail element c > b of N+(a) streamed, 4 B per N+(b) entry staged
+    # (+ its c(b, x) flush), 8 B per triangle (the c(a, c) reduction); merge
+    # part -- per heavy-middle edge 40 B + 4 B per merged out-list entry
+    CAP = 4096
+    a_o = rows[up]
+    b_o = adj_h[up].astype(np.int64)
+    oofs_h = np.concatenate([[0], np.cumsum(out)]).astype(np.int64)
+    tail = out[a_o] - (np.arange(len(a_o), dtype=np.int64) - oofs_h[a_o]) - 1
+    ob = out[b_o]
+    light = (ob >= 1) & (ob <= CAP)
+    heavy = ob > CAP
+    tri = 0
+    if plan is not None and plan.support() is not None:
+        tri = int(plan.support().to(torch.int64).sum().item()) // 3
+    mid = (out >= 1) & (out <= CAP) & (indeg >= 1)
+    sup_bytes = (32.0 * float(light.sum()) + 4.0 * float(tail[light].sum()) + 8.0 * float(out[mid].sum())
+                 + 8.0 * tri + 40.0 * float(heavy.sum()) + 4.0 * float((out[a_o] + ob)[heavy].sum()))
     # fc pass: per root edge 8 B (u,v) + 32 B (4 offsets) + 4 B support
     fc_bytes = 44.0 * m * share
     # general / triangle core passes: compulsory graph bytes (CSR + oriented

@@ -463,6 +463,246 @@ __global__ void __launch_bounds__(256) support_kernel(GraphDev G, OrientDev O, i
     }
 }
 
+// Wedge-hash part of the support pass: every triangle a < b < c is found
+// from its MIDDLE vertex b.  A warp takes a unit (b, k) from a global atomic
+// queue, stages N+(b) (out(b) <= FSGC_SUP_CAP) in a shared-memory hash table
+// (key -> position in N+(b)), takes the k-th slice of b's in-list
+// N-(b) = {a < b}, and streams, for every a of the slice, the tail of N+(a)
+// after b (the c > b; b's position in N+(a) comes from graph.rev), probing
+// each c in the table.  The tails of the slice are concatenated (warp prefix
+// sum of their lengths) so the 32 lanes always read 32 consecutive virtual
+// elements: coalesced adjacency reads whatever the tail lengths.  A hit is
+// the triangle (a, b, c): c(bc) += 1 in shared memory (flushed per unit),
+// c(ab) += 1 in shared memory (flushed per slice), c(ac) += 1 by a global
+// reduction.  Work: sum_a out(a)^2 / 2 adjacency elements instead of the
+// merge's sum_(a,b) (out(a) + out(b)).
+// Two variants: a small table (out(b) <= CAPW, the many small middles; the
+// slice's tails are concatenated, sup_slice) and a large one (CAPW < out(b)
+// <= CAP: long tails, streamed one at a time, sup_slice_stream).  One warp
+// per unit, its own table sized to out(b) (load factor <= 1/2), no block
+// barriers.
+template <int CAPT>
+struct SupLayout {
+    static constexpr bool STREAM = CAPT > FSGC_SUP_CAPW;
+    static constexpr int WARPS = STREAM ? 4 : 8;
+    static constexpr int HS = 2 * CAPT;
+    static constexpr size_t table_bytes = (size_t)HS * 4 + (size_t)HS * 2 + (size_t)CAPT * 4;
+    static constexpr size_t slice_bytes = STREAM ? 0 : (size_t)(FSGC_SUP_SEG + 4) * 4 + (size_t)4 * FSGC_SUP_SEG * 4;
+    static constexpr size_t warp_bytes = table_bytes + slice_bytes;
+    static constexpr size_t bytes = WARPS * warp_bytes;
+};
+
+// one warp, one slice [ib0, ib0 + len) of N-(b): tails of N+(a) after b,
+// concatenated; two virtual elements per lane in flight
+__device__ __forceinline__ void sup_slice(const GraphDev& G, const OrientDev& O, const int32_t* __restrict__ rev,
+                                          int* __restrict__ sup, int64_t ib0, int len, int64_t rbase,
+                                          const int32_t* key, const int16_t* kpos, int32_t* cb, int hbits,
+                                          int32_t* pre, uint32_t* q0, uint32_t* da, int32_t* ea, int32_t* cab,
+                                          int lane) {
+    const uint32_t hm = (1u << hbits) - 1;
+    int carry = 0;
+    for (int j0 = 0; j0 < len; j0 += 32) {
+        const int j = j0 + lane;
+        int L = 0;
+        if (j < len) {
+            const int a = __ldg(G.adj + ib0 + j);
+            const int e = __ldg(rev + rbase + j);
+            const int64_t sa = __ldg(O.split + a), oa = __ldg(O.oofs + a);
+            const int64_t q = sa + (e - oa) + 1;
+            L = (int)(__ldg(G.offs + a + 1) - q);
+            q0[j] = (uint32_t)q;
+            da[j] = (uint32_t)(sa - oa);
+            ea[j] = e;
+            cab[j] = 0;
+        }
+        int x = L;                        // inclusive warp scan
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(FULLMASK, x, o);
+            if (lane >= o) x += y;
+        }
+        if (j < len) pre[j] = carry + x - L;
+        carry += __shfl_sync(FULLMASK, x, 31);
+    }
+    if (lane == 0) pre[len] = carry;
+    __syncwarp();
+    const int total = carry;
+    int lo = 0;                           // monotone: last j with pre[j] <= idx
+    for (int v0 = 0; v0 < total; v0 += 64) {
+        int jj[2], cc[2];
+        uint32_t pp[2];
+        bool ok[2];
+#pragma unroll
+        for (int r = 0; r < 2; ++r) {
+            const int idx = v0 + 32 * r + lane;
+            ok[r] = idx < total;
+            jj[r] = 0; pp[r] = 0; cc[r] = -1;
+            if (ok[r]) {
+                int l2 = lo, hi = len;
+                while (hi - l2 > 1) {
+                    const int mid = (l2 + hi) >> 1;
+                    if (pre[mid] <= idx) l2 = mid; else hi = mid;
+                }
+                lo = l2;
+                jj[r] = l2;
+                pp[r] = q0[l2] + (uint32_t)(idx - pre[l2]);
+                cc[r] = __ldg(G.adj + pp[r]);
+            }
+        }
+#pragma unroll
+        for (int r = 0; r < 2; ++r) {
+            bool hit = false;
+            int kk = -1;
+            if (ok[r]) {
+                uint32_t h = ((uint32_t)cc[r] * 0x9E3779B1u) >> (32 - hbits);
+                int y;
+                while ((y = key[h]) != cc[r] && y != -1) h = (h + 1) & hm;
+                hit = y == cc[r];
+                if (hit) kk = kpos[h];
+            }
+            const unsigned hmask = __ballot_sync(FULLMASK, hit);
+            if (hit) {
+                atomicAdd(&cb[kk], 1);
+                atomicAdd(sup + (pp[r] - da[jj[r]]), 1);
+                const unsigned peers = __match_any_sync(hmask, jj[r]);   // c(a, b): one add per a
+                if ((peers & ((1u << lane) - 1)) == 0) atomicAdd(&cab[jj[r]], __popc(peers));
+            }
+        }
+    }
+    __syncwarp();
+    for (int j = lane; j < len; j += 32)
+        if (cab[j]) atomicAdd(sup + ea[j], cab[j]);
+    __syncwarp();
+}
+
+constexpr int kSupILP = 4;   // tail loads in flight per lane
+
+// one warp, one slice of N-(b) whose tails are long (block tables: the
+// middles of large out-degree): the warp streams one tail at a time, 32
+// consecutive elements per step (two steps in flight), c(a, b) = the hits
+// counted by ballot, one global add per (a, b)
+__device__ __forceinline__ void sup_slice_stream(const GraphDev& G, const OrientDev& O,
+                                                 const int32_t* __restrict__ rev, int* __restrict__ sup,
+                                                 int64_t ib0, int len, int64_t rbase, const int32_t* key,
+                                                 const int16_t* kpos, int32_t* cb, int hbits, int lane) {
+    const uint32_t hm = (1u << hbits) - 1;
+    for (int j0 = 0; j0 < len; j0 += 32) {
+        const int j = j0 + lane;
+        int64_t q = 0, dA = 0;
+        int L = 0, e = 0;
+        if (j < len) {
+            const int a = __ldg(G.adj + ib0 + j);
+            e = __ldg(rev + rbase + j);
+            const int64_t sa = __ldg(O.split + a), oa = __ldg(O.oofs + a);
+            q = sa + (e - oa) + 1;
+            L = (int)(__ldg(G.offs + a + 1) - q);
+            dA = sa - oa;
+        }
+        const int nj = min(32, len - j0);
+        for (int t = 0; t < nj; ++t) {
+            const int64_t qt = __shfl_sync(FULLMASK, q, t);
+            const int Lt = __shfl_sync(FULLMASK, L, t);
+            const int64_t dt = __shfl_sync(FULLMASK, dA, t);
+            int hits = 0;
+            for (int o0 = 0; o0 < Lt; o0 += 32 * kSupILP) {
+                int cc[kSupILP];
+#pragma unroll
+                for (int r = 0; r < kSupILP; ++r) {
+                    const int o = o0 + 32 * r + lane;
+                    cc[r] = o < Lt ? __ldg(G.adj + qt + o) : -1;
+                }
+#pragma unroll
+                for (int r = 0; r < kSupILP; ++r) {
+                    bool hit = false;
+                    if (cc[r] >= 0) {
+                        uint32_t h = ((uint32_t)cc[r] * 0x9E3779B1u) >> (32 - hbits);
+                        int y;
+                        while ((y = key[h]) != cc[r] && y != -1) h = (h + 1) & hm;
+                        if (y == cc[r]) {
+                            hit = true;
+                            atomicAdd(&cb[kpos[h]], 1);
+                            atomicAdd(sup + (qt + o0 + 32 * r + lane - dt), 1);
+                        }
+                    }
+                    hits += __popc(__ballot_sync(FULLMASK, hit));
+                }
+            }
+            const int et = __shfl_sync(FULLMASK, e, t);
+            if (lane == 0 && hits) atomicAdd(sup + et, hits);
+        }
+    }
+}
+
+template <int CAPT>
+__global__ void __launch_bounds__(SupLayout<CAPT>::WARPS * 32, 1) support_hash_kernel(
+    GraphDev G, OrientDev O, const int32_t* __restrict__ rev, const uint64_t* __restrict__ units, int64_t nunits,
+    int* __restrict__ sup, unsigned long long* queue, int shard, int nshards) {
+    typedef SupLayout<CAPT> Lay;
+    extern __shared__ __align__(16) unsigned char s_sup[];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    unsigned char* tb = s_sup + w * Lay::warp_bytes;
+    int32_t* key = reinterpret_cast<int32_t*>(tb);
+    int16_t* kpos = reinterpret_cast<int16_t*>(tb + (size_t)Lay::HS * 4);
+    int32_t* cb = reinterpret_cast<int32_t*>(tb + (size_t)Lay::HS * 6);
+    unsigned char* wb = tb + Lay::table_bytes;
+    int32_t* pre = reinterpret_cast<int32_t*>(wb);
+    uint32_t* q0 = reinterpret_cast<uint32_t*>(wb + (FSGC_SUP_SEG + 4) * 4);
+    uint32_t* da = q0 + FSGC_SUP_SEG;
+    int32_t* ea = reinterpret_cast<int32_t*>(da + FSGC_SUP_SEG);
+    int32_t* cab = ea + FSGC_SUP_SEG;
+    int prev_b = -1, ob = 0, hbits = 5;
+    int64_t sb = 0;
+    const int64_t mine = nunits > shard ? (nunits - shard + nshards - 1) / nshards : 0;
+    for (;;) {
+        unsigned long long jq = 0;
+        if (lane == 0) jq = atomicAdd(queue, 1ull);
+        jq = __shfl_sync(FULLMASK, jq, 0);
+        if ((int64_t)jq >= mine) break;
+        // large tables: the largest middles (end of the degree order) first
+        const int64_t t = (int64_t)jq * nshards + shard;
+        const uint64_t un = __ldg(units + (Lay::STREAM ? nunits - 1 - t : t));
+        const int b = (int)(un >> 32), k = (int)(un & 0xffffffffu);
+        if (b != prev_b) {                    // (re)build the table of N+(b)
+            if (prev_b >= 0) {                // flush c(b', x) of the previous b'
+                const int64_t base = __ldg(O.oofs + prev_b);
+                for (int i = lane; i < ob; i += 32)
+                    if (cb[i]) atomicAdd(sup + base + i, cb[i]);
+            }
+            sb = __ldg(O.split + b);
+            ob = (int)(__ldg(G.offs + b + 1) - sb);
+            hbits = 5;
+            while ((1 << hbits) < 2 * ob) ++hbits;
+            __syncwarp();
+            for (int i = lane; i < (1 << hbits); i += 32) key[i] = -1;
+            for (int i = lane; i < ob; i += 32) cb[i] = 0;
+            __syncwarp();
+            const uint32_t hm = (1u << hbits) - 1;
+            for (int i = lane; i < ob; i += 32) {
+                const int x = __ldg(G.adj + sb + i);
+                uint32_t h = ((uint32_t)x * 0x9E3779B1u) >> (32 - hbits);
+                while (atomicCAS(&key[h], -1, x) != -1) h = (h + 1) & hm;
+                kpos[h] = (int16_t)i;
+            }
+            prev_b = b;
+            __syncwarp();
+        }
+        const int64_t ib0 = __ldg(G.offs + b) + (int64_t)k * FSGC_SUP_SEG;
+        const int len = (int)min((int64_t)FSGC_SUP_SEG, sb - ib0);
+        const int64_t rbase = ib0 - __ldg(O.oofs + b);
+        if (Lay::STREAM)
+            sup_slice_stream(G, O, rev, sup, ib0, len, rbase, key, kpos, cb, hbits, lane);
+        else
+            sup_slice(G, O, rev, sup, ib0, len, rbase, key, kpos, cb, hbits, pre, q0, da, ea, cab, lane);
+        __syncwarp();
+    }
+    if (prev_b >= 0) {
+        __syncwarp();
+        const int64_t base = __ldg(O.oofs + prev_b);
+        for (int i = lane; i < ob; i += 32)
+            if (cb[i]) atomicAdd(sup + base + i, cb[i]);
+    }
+}
+
 // One program of the Sec. 3.1 closed form, out of line: the kernels are short
 // and latency-bound, so a compact hot path (instruction-cache footprint)
 // matters more than call overhead.  `small`: the 64-bit bound holds.
@@ -1747,8 +1987,10 @@ struct fsgc_plan {
     // one per-edge support array c(e) = |N(u) & N(v)| for every pass that
     // reads it (edge, triangle and general cores), at ws[sup_off, + 4 m)
     int sup_first = -1;            // first pass reading it (-1: none)
-    size_t sup_off = 0;
-    int64_t grid_sup = 1;
+    size_t sup_off = 0;            // the array; its work-queue counter 256 bytes before
+    int64_t grid_sup = 1;          // merge part (heavy middle vertices)
+    int64_t grid_hash = 1;         // wedge-hash part, warp tables
+    int64_t grid_hash_big = 1;     // wedge-hash part, block tables
     int sup_shard = 0, sup_nshards = 1;   // FSGC_FLAG_SHARD_SUPPORT: this shard's part
     std::vector<cudaEvent_t> ev;   // support begin/end, then begin/end per pass
     unsigned long long* trace = nullptr;
@@ -1840,10 +2082,18 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
         P->passes.push_back(X);
     }
     if (P->sup_first >= 0) {
-        P->sup_off = off;
-        off += ((size_t)g->m * sizeof(int) + 255) & ~(size_t)255;
+        P->sup_off = off + 256;
+        off += 256 + (((size_t)g->m * sizeof(int) + 255) & ~(size_t)255);
         P->grid_sup = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy((const void*)support_kernel, 256, 0),
-                                                             (g->m + 255) / 256));
+                                                             (g->nsup_heavy + 255) / 256));
+        typedef SupLayout<FSGC_SUP_CAPW> LS;
+        typedef SupLayout<FSGC_SUP_CAP> LB;
+        P->grid_hash = std::max<int64_t>(1, std::min<int64_t>(
+            (int64_t)nsm * occupancy((const void*)support_hash_kernel<FSGC_SUP_CAPW>, LS::WARPS * 32, LS::bytes),
+            (g->nsup_units + LS::WARPS - 1) / LS::WARPS));
+        P->grid_hash_big = std::max<int64_t>(1, std::min<int64_t>(
+            (int64_t)nsm * occupancy((const void*)support_hash_kernel<FSGC_SUP_CAP>, LB::WARPS * 32, LB::bytes),
+            (g->nsup_units_big + LB::WARPS - 1) / LB::WARPS));
         if ((opts.flags & FSGC_FLAG_SHARD_SUPPORT) && opts.shard_count > 1) {
             P->sup_shard = opts.shard_index;
             P->sup_nshards = opts.shard_count;
@@ -1958,12 +2208,35 @@ extern "C" int fsgc_plan_enqueue_stage(const fsgc_plan* P, void* workspace, void
     OrientDev O{g->split, g->oofs};
     int* dsup = (int*)((unsigned char*)workspace + P->sup_off);
     if ((stages & FSGC_STAGE_SUPPORT) && P->sup_first >= 0) {   // (A) per-edge common-neighbour counts
-        FSGC_CUDA(cudaMemsetAsync(dsup, 0, (size_t)g->m * sizeof(int), st));
+        unsigned long long* dq = (unsigned long long*)((unsigned char*)dsup - 256);   // 2 queue counters
+        FSGC_CUDA(cudaMemsetAsync(dq, 0, 256 + (size_t)g->m * sizeof(int), st));
         FSGC_CUDA(cudaEventRecordWithFlags(P->ev[0], st, evflags));
-        support_kernel<<<(int)P->grid_sup, 256, 0, st>>>(G, O, g->m, dsup, g->sorder, g->ssrc, g->sdst,
-                                                          P->sup_shard, P->sup_nshards,
-                                                          P->trace ? P->trace + (1 << 17) : nullptr);
-        FSGC_CUDA(cudaGetLastError());
+        // FSGC_SUP_MERGE_ONLY=1 (experiments): the merge kernel over every
+        // oriented edge (the work list holds the light ones after the heavy)
+        const bool merge_only = tune("FSGC_SUP_MERGE_ONLY", 0) != 0;
+        if (g->nsup_units_big > 0 && !merge_only) {
+            typedef SupLayout<FSGC_SUP_CAP> LB;
+            support_hash_kernel<FSGC_SUP_CAP><<<(int)P->grid_hash_big, LB::WARPS * 32, LB::bytes, st>>>(
+                G, O, g->rev, g->sup_units_big, g->nsup_units_big, dsup, dq + 1, P->sup_shard, P->sup_nshards);
+            FSGC_CUDA(cudaGetLastError());
+        }
+        if (g->nsup_units > 0 && !merge_only) {
+            typedef SupLayout<FSGC_SUP_CAPW> LS;
+            support_hash_kernel<FSGC_SUP_CAPW><<<(int)P->grid_hash, LS::WARPS * 32, LS::bytes, st>>>(
+                G, O, g->rev, g->sup_units, g->nsup_units, dsup, dq, P->sup_shard, P->sup_nshards);
+            FSGC_CUDA(cudaGetLastError());
+        }
+        const int64_t nmerge = merge_only ? g->m : g->nsup_heavy;
+        if (nmerge > 0) {
+            const int grid = merge_only ? (int)std::max<int64_t>(P->grid_sup, std::min<int64_t>(
+                                              (int64_t)sm_count() * occupancy((const void*)support_kernel, 256, 0),
+                                              (g->m + 255) / 256))
+                                        : (int)P->grid_sup;
+            support_kernel<<<grid, 256, 0, st>>>(G, O, nmerge, dsup, g->sorder, g->ssrc,
+                                                              g->sdst, P->sup_shard, P->sup_nshards,
+                                                              P->trace ? P->trace + (1 << 17) : nullptr);
+            FSGC_CUDA(cudaGetLastError());
+        }
         FSGC_CUDA(cudaEventRecordWithFlags(P->ev[1], st, evflags));
     }
     if (!(stages & FSGC_STAGE_COUNT)) return FSGC_OK;
@@ -2027,7 +2300,9 @@ extern "C" int fsgc_plan_decode(const fsgc_plan* P, const void* raw, fsgc_result
         if (sup_here && cudaEventElapsedTime(&ams, P->ev[0], P->ev[1]) != cudaSuccess) ams = -1.f;
         if (cudaEventElapsedTime(&kms, P->ev[2 + 2 * pi], P->ev[3 + 2 * pi]) != cudaSuccess) kms = -1.f;
         cudaGetLastError();   // timing is best effort (e.g. events recorded inside a graph)
-        const int launches = (X.W.end > X.W.begin ? 1 : 0) + (sup_here ? 1 : 0);
+        const int launches = (X.W.end > X.W.begin ? 1 : 0) +
+                             (sup_here ? (P->g->nsup_units > 0 ? 1 : 0) + (P->g->nsup_units_big > 0 ? 1 : 0) +
+                                             (P->g->nsup_heavy > 0 ? 1 : 0) : 0);
         for (size_t mi = 0; mi < X.plan.members.size(); ++mi) {
             fsgc_result& r = results[X.plan.members[mi]];
             r.raw.lo = acc[mi].lo;

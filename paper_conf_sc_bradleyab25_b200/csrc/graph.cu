@@ -144,19 +144,62 @@ struct UpperTri {
     __host__ __device__ bool operator()(const uint64_t& k) const { return (k >> B) < (k & mask); }
 };
 
-// support-pass work order: key = merge length out(u) + out(v) of oriented
-// edge i (capped), value = i; sorted, so the 32 lanes of a warp get roots of
-// similar cost (degree-aware binning, north_star)
+// merge-part work order: key = merge length out(u) + out(v) of oriented
+// edge i (capped) when its middle vertex v has out(v) > FSGC_SUP_CAP, else
+// the maximum key (sorted to the end, not used); value = i; sorted, so the 32
+// lanes of a warp get roots of similar cost (degree-aware binning, north_star)
 __global__ void support_work_keys(const int64_t* __restrict__ offs, const int64_t* __restrict__ split,
                                   const int32_t* __restrict__ osrc, const int32_t* __restrict__ odst, int64_t m,
-                                  uint32_t* __restrict__ key, int32_t* __restrict__ idx) {
+                                  uint32_t* __restrict__ key, int32_t* __restrict__ idx,
+                                  unsigned long long* nheavy, int64_t cap) {
+    int cnt = 0;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m;
          i += (int64_t)gridDim.x * blockDim.x) {
         const int u = osrc[i], v = odst[i];
-        const int64_t w = (offs[u + 1] - split[u]) + (offs[v + 1] - split[v]);
-        key[i] = (uint32_t)(w < (1 << 20) ? w : (1 << 20) - 1);
+        const int64_t ov = offs[v + 1] - split[v];
+        const int64_t w = (offs[u + 1] - split[u]) + ov;
+        const bool heavy = ov > cap;
+        key[i] = heavy ? (uint32_t)(w < (1 << 20) - 1 ? w : (1 << 20) - 2) : (uint32_t)((1 << 20) - 1);
         idx[i] = (int32_t)i;
+        cnt += heavy;
     }
+    if (cnt) atomicAdd(nheavy, (unsigned long long)cnt);
+}
+
+// rev[i - oofs[b]] = oriented index of (a, b) for the in-entry a = adj[i] of
+// row b: sorting the oriented edges (a, b), stored in (a, b) order, by
+// (b, a) lists them in the in-entries' CSR order.  Keys b << B | a, values e.
+__global__ void rev_keys(const int32_t* __restrict__ osrc, const int32_t* __restrict__ odst, int64_t m, int B,
+                         uint64_t* __restrict__ key, int32_t* __restrict__ val) {
+    for (int64_t e = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; e < m;
+         e += (int64_t)gridDim.x * blockDim.x) {
+        key[e] = ((uint64_t)odst[e] << B) | (uint64_t)osrc[e];
+        val[e] = (int32_t)e;
+    }
+}
+
+// wedge-hash units per middle vertex b (cnt[n] = 0 for the scans):
+// small-table units ceil(in(b) / SEG) when 1 <= out(b) <= CAPW, large-table
+// units ceil(in(b) / SEG) when CAPW < out(b) <= CAP
+__global__ void unit_counts(const int64_t* __restrict__ offs, const int64_t* __restrict__ split, int64_t n,
+                            int64_t* __restrict__ cnt, int64_t* __restrict__ cnt_big) {
+    for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b <= n;
+         b += (int64_t)gridDim.x * blockDim.x) {
+        int64_t c = 0, cb = 0;
+        if (b < n) {
+            const int64_t in = split[b] - offs[b], out = offs[b + 1] - split[b];
+            if (in >= 1 && out >= 1 && out <= FSGC_SUP_CAPW) c = (in + FSGC_SUP_SEG - 1) / FSGC_SUP_SEG;
+            if (in >= 1 && out > FSGC_SUP_CAPW && out <= FSGC_SUP_CAP) cb = (in + FSGC_SUP_SEG - 1) / FSGC_SUP_SEG;
+        }
+        cnt[b] = c;
+        cnt_big[b] = cb;
+    }
+}
+
+__global__ void unit_fill(const int64_t* __restrict__ uofs, int64_t n, uint64_t* __restrict__ units) {
+    for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b < n;
+         b += (int64_t)gridDim.x * blockDim.x)
+        for (int64_t k = uofs[b]; k < uofs[b + 1]; ++k) units[k] = ((uint64_t)b << 32) | (uint64_t)(k - uofs[b]);
 }
 
 __global__ void gather_uv(const int32_t* __restrict__ idx, const int32_t* __restrict__ osrc,
@@ -366,8 +409,51 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
         if (b > tmp_bytes) { FSGC_CUDA(tmp.alloc(b, st)); tmp_bytes = b; }
         FSGC_CUDA(cub::DeviceScan::ExclusiveSum(tmp.ptr, b, oofs.ptr, oofs.ptr, n + 1, st));
     }
-    // support-pass order (sorted by merge length) with its (u, v) gathered
-    DevBuf<int32_t> sorder, ssrc, sdst;
+    // support pass, merge part: heavy-middle edges sorted by merge length
+    // with their (u, v) gathered; wedge-hash part: rev index + units
+    DevBuf<int32_t> sorder, ssrc, sdst, rev;
+    DevBuf<uint64_t> units, units_big;
+    DevBuf<int64_t> ucnt, ucnt_big;
+    FSGC_CUDA(cudaMemsetAsync(dnum.ptr, 0, 2 * sizeof(int64_t), st));
+    // small graphs (launch-latency bound): the merge part alone, over every
+    // edge (FSGC_SUP_HASH_MIN_M overrides the threshold)
+    int64_t hash_min_m = 1 << 20;
+    if (const char* v = getenv("FSGC_SUP_HASH_MIN_M")) hash_min_m = atoll(v);
+    const bool use_hash = m >= hash_min_m;
+    if (m > 0 && use_hash) {
+        {   // rev = oriented edge ids in (b, a) order = the in-entries' CSR order
+            DevBuf<uint64_t> rk0, rk1;
+            DevBuf<int32_t> rv1;
+            FSGC_CUDA(rk0.alloc(m, st));
+            FSGC_CUDA(rk1.alloc(m, st));
+            FSGC_CUDA(rev.alloc(m, st));
+            FSGC_CUDA(rv1.alloc(m, st));
+            rev_keys<<<grid_for(m), 256, 0, st>>>(osrc.ptr, odst.ptr, m, B, rk0.ptr, rev.ptr);
+            FSGC_CUDA(cudaGetLastError());
+            cub::DoubleBuffer<uint64_t> dk(rk0.ptr, rk1.ptr);
+            cub::DoubleBuffer<int32_t> dv(rev.ptr, rv1.ptr);
+            size_t b = 0;
+            FSGC_CUDA(cub::DeviceRadixSort::SortPairs(nullptr, b, dk, dv, m, 0, keybits, st));
+            if (b > tmp_bytes) { FSGC_CUDA(tmp.alloc(b, st)); tmp_bytes = b; }
+            FSGC_CUDA(cub::DeviceRadixSort::SortPairs(tmp.ptr, b, dk, dv, m, 0, keybits, st));
+            if (dv.Current() != rev.ptr) std::swap(rev.ptr, rv1.ptr);
+        }
+        FSGC_CUDA(ucnt.alloc(n + 1, st));
+        FSGC_CUDA(ucnt_big.alloc(n + 1, st));
+        unit_counts<<<grid_for(n + 1), 256, 0, st>>>(offs.ptr, split.ptr, n, ucnt.ptr, ucnt_big.ptr);
+        FSGC_CUDA(cudaGetLastError());
+        size_t b = 0;
+        FSGC_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, b, ucnt.ptr, ucnt.ptr, n + 1, st));
+        if (b > tmp_bytes) { FSGC_CUDA(tmp.alloc(b, st)); tmp_bytes = b; }
+        FSGC_CUDA(cub::DeviceScan::ExclusiveSum(tmp.ptr, b, ucnt.ptr, ucnt.ptr, n + 1, st));
+        FSGC_CUDA(cub::DeviceScan::ExclusiveSum(tmp.ptr, b, ucnt_big.ptr, ucnt_big.ptr, n + 1, st));
+        FSGC_CUDA(units.alloc((size_t)n + (size_t)m / FSGC_SUP_SEG + 1, st));   // >= sum ceil(in/SEG)
+        FSGC_CUDA(units_big.alloc((size_t)m / FSGC_SUP_CAPW + (size_t)m / FSGC_SUP_SEG + 1, st));
+        unit_fill<<<grid_for(n), 256, 0, st>>>(ucnt.ptr, n, units.ptr);
+        FSGC_CUDA(cudaGetLastError());
+        unit_fill<<<grid_for(n), 256, 0, st>>>(ucnt_big.ptr, n, units_big.ptr);
+        FSGC_CUDA(cudaGetLastError());
+    }
     if (m > 0) {
         DevBuf<uint32_t> k0, k1;
         DevBuf<int32_t> i1;
@@ -375,7 +461,9 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
         FSGC_CUDA(k1.alloc(m, st));
         FSGC_CUDA(sorder.alloc(m, st));
         FSGC_CUDA(i1.alloc(m, st));
-        support_work_keys<<<grid_for(m), 256, 0, st>>>(offs.ptr, split.ptr, osrc.ptr, odst.ptr, m, k0.ptr, sorder.ptr);
+        support_work_keys<<<grid_for(m), 256, 0, st>>>(offs.ptr, split.ptr, osrc.ptr, odst.ptr, m, k0.ptr, sorder.ptr,
+                                                       (unsigned long long*)dnum.ptr,
+                                                       use_hash ? (int64_t)FSGC_SUP_CAP : (int64_t)-1);
         FSGC_CUDA(cudaGetLastError());
         cub::DoubleBuffer<uint32_t> dk(k0.ptr, k1.ptr);
         cub::DoubleBuffer<int32_t> dv(sorder.ptr, i1.ptr);
@@ -398,6 +486,7 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
     // memory); FSGC_HUB_BYTES overrides), only for degree >= kHubMinDeg
     int64_t hub_base = n, hub_words = (n + 31) / 32;
     int64_t maxdeg = 0;   // the last vertex has the largest degree
+    int64_t nheavy = 0, nunits = 0, nunits_big = 0;
     DevBuf<uint32_t> hubs;
     {
         size_t free_b = 0, total_b = 0;
@@ -411,11 +500,18 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
         // first v in [n - max_hubs, n) with deg(v) >= kHubMinDeg (degrees are
         // ascending in the new ids), and the maximum degree: one synchronisation
         int64_t hv2[2] = {n, 0};
+        if (m > 0) FSGC_CUDA(cudaMemcpyAsync(&nheavy, dnum.ptr, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+        if (m > 0 && use_hash) {   // heavy-edge count (dnum[0], from support_work_keys) and units
+            FSGC_CUDA(cudaMemcpyAsync(&nunits, ucnt.ptr + n, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+            FSGC_CUDA(cudaMemcpyAsync(&nunits_big, ucnt_big.ptr + n, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+        }
         if (n > 0) {
+            DevBuf<int64_t> hs;
+            FSGC_CUDA(hs.alloc(2, st));
             hub_search<<<1, 1, 0, st>>>(offs.ptr, n, n - std::max<int64_t>(0, std::min<int64_t>(max_hubs, n)),
-                                        M > 0 ? 256 : (int64_t)1 << 62, dnum.ptr);
+                                        M > 0 ? 256 : (int64_t)1 << 62, hs.ptr);
             FSGC_CUDA(cudaGetLastError());
-            FSGC_CUDA(cudaMemcpyAsync(hv2, dnum.ptr, 2 * sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+            FSGC_CUDA(cudaMemcpyAsync(hv2, hs.ptr, 2 * sizeof(int64_t), cudaMemcpyDeviceToHost, st));
             FSGC_CUDA(cudaStreamSynchronize(st));
         }
         if (max_hubs > 0 && M > 0) hub_base = hv2[0];
@@ -446,6 +542,12 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
     g->sorder = sorder.take();
     g->ssrc = ssrc.take();
     g->sdst = sdst.take();
+    g->nsup_heavy = nheavy;
+    g->sup_units = units.take();
+    g->nsup_units = nunits;
+    g->sup_units_big = units_big.take();
+    g->nsup_units_big = nunits_big;
+    g->rev = rev.take();
     g->hub_base = hub_base;
     g->hub_words = hub_words;
     g->hub_bits = hubs.take();
@@ -489,6 +591,9 @@ extern "C" void fsgc_free_graph(fsgc_graph* g) {
     cudaFree(g->sorder);
     cudaFree(g->ssrc);
     cudaFree(g->sdst);
+    cudaFree(g->sup_units);
+    cudaFree(g->sup_units_big);
+    cudaFree(g->rev);
     cudaFree(g->hub_bits);
     delete g;
 }

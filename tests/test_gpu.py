@@ -439,3 +439,24 @@ def test_k_tailed_triangles_rmat16_closed_form():
         want = oracle.k_tailed_triangles(gadj, k)
         assert not batch[k - 1].overflow and batch[k - 1].count == want, k
         assert F.fsgc_count(g, [pats[k - 1]])[0].count == want, k
+
+
+@pytest.mark.parametrize("wl", ["rmat16", "pl2k"])
+def test_wedge_hash_support_equals_merge(wl, monkeypatch):
+    """The support pass's two algorithms -- the wedge-hash kernels (middle
+    vertex tables; forced with FSGC_SUP_HASH_MIN_M=0) and the merge kernel
+    (graphs below the threshold) -- give the identical int32[m] support array
+    and identical counts (edge, triangle and 4-clique cores)."""
+    n, e, _ = workload(wl)
+    names = ["2-tailed-triangle", "tricore+3f", "k4core+2f"]
+    pats = [F.compile_named(PATTERNS[x]) for x in names]
+    out = []
+    for thr in ("0", str(1 << 40)):
+        monkeypatch.setenv("FSGC_SUP_HASH_MIN_M", thr)
+        g = F.fsgc_load_graph(e, n)
+        plan = F.Plan(g, pats)
+        plan.enqueue()
+        torch.cuda.synchronize()
+        out.append((plan.support().clone(), [r.raw for r in plan.decode()]))
+    assert torch.equal(out[0][0], out[1][0])
+    assert out[0][1] == out[1][1]
