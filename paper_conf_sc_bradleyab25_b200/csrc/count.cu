@@ -942,6 +942,7 @@ struct VennDev {
     int32_t n;                   // terms; 0: table off (per-program Listing 5)
     int32_t nrows;               // row entries per core match (C(n_r, j), j >= 1)
     float slack;                 // log2(programs per pattern) + margin
+    int32_t warp;                // 1: one diagram per warp (large tables), 0: one per lane
     uint8_t maxs[64];            // per region: max s_r (0: no row)
     uint8_t base[64];            // per region: first row entry
 };
@@ -1005,6 +1006,98 @@ __device__ __forceinline__ void venn_terms_eval(const uint32_t* venn, int V, con
         sum += pr;
     }
     acc.add(cur, (u128)sum, false);
+}
+
+// The same table, one diagram per WARP: the lanes owning a region build its
+// binomial row in the warp's shared buffer, then take the terms strided (each
+// lane's subsequence stays grouped by pattern, and its partial sums are
+// bounded by the pattern's sum, so the tier argument above holds per lane).
+template <class W, int NP>
+__device__ __forceinline__ void venn_warp_terms(const uint32_t* venn, int V, const VennDev& T, W* R, int lane,
+                                                AccN<NP>& acc) {
+    for (int r = 1 + lane; r < V; r += 32) {
+        const int K = T.maxs[r];
+        if (!K) continue;
+        const uint64_t n = venn[r];
+        W* Rr = R + T.base[r];
+        W c = 1;
+        for (int j = 1; j <= K; ++j) {
+            c = ((c * (W)(n - (uint64_t)j + 1)) >> c_tz[j]) * inv_odd(j, c);
+            Rr[j - 1] = c;
+        }
+    }
+    __syncwarp();
+    W sum = 0;
+    int cur = -1;
+    for (int t = lane; t < T.n; t += 32) {
+        const VTerm* e = T.terms + t;
+        const uint64_t cf = __ldg(&e->coef);
+        const uint2 hd = __ldg(reinterpret_cast<const uint2*>(e) + 1);
+        const uint2 tl = __ldg(reinterpret_cast<const uint2*>(e) + 2);
+        const int pat = hd.x & 255, nz = (hd.x >> 8) & 255;
+        if (pat != cur) {
+            if (cur >= 0) acc.add(cur, (u128)sum, false);
+            sum = 0;
+            cur = pat;
+        }
+        W pr = (W)cf;
+        const uint32_t words[4] = {hd.x >> 16, hd.y, tl.x, tl.y};
+#pragma unroll
+        for (int i = 0; i < kMaxVennNz; ++i) {
+            if (i >= nz) break;
+            const int o = i < 2 ? (int)((words[0] >> (8 * i)) & 255)
+                                : (int)((words[1 + (i - 2) / 4] >> (8 * ((i - 2) & 3))) & 255);
+            pr *= R[o];
+        }
+        sum += pr;
+    }
+    if (cur >= 0) acc.add(cur, (u128)sum, false);
+    __syncwarp();
+}
+
+// venn_bound_log2 with the programs split over the lanes (warp max)
+__device__ __forceinline__ float venn_bound_log2_warp(const uint32_t* venn, int q, const CoreProg& P, int lane) {
+    const int V = 1 << q;
+    float lz[64];
+    {
+        uint32_t Z[64];
+        for (int A = 0; A < V; ++A) Z[A] = A ? venn[A] : 0;
+        for (int bb = 0; bb < q; ++bb)
+            for (int A = 0; A < V; ++A)
+                if (!(A >> bb & 1)) Z[A] += Z[A | (1 << bb)];
+        for (int A = 0; A < V; ++A) lz[A] = log2f((float)Z[A] + 1.f);
+    }
+    float mx = 0.f;
+    for (int pi = lane; pi < P.nprog; pi += 32) {
+        const FringeProg& fp = P.prog[pi];
+        float b = 0.f;
+        for (int t = 0; t < fp.s; ++t) b += (float)fp.k[t] * lz[fp.anch[t]];
+        mx = fmaxf(mx, b);
+    }
+#pragma unroll
+    for (int o = 16; o; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(FULLMASK, mx, o));
+    return mx;
+}
+
+// fc of one diagram by the whole warp: table tiers, else checked Listing 5
+// with the programs split over the lanes
+template <int STACK, int NP>
+__device__ __forceinline__ void venn_fc_warp(uint32_t* vloc, int q, const CoreProg& P, const VennDev& VD,
+                                             u128* rows, int lane, AccN<NP>& acc) {
+    const int V = 1 << q;
+    const float bnd = venn_bound_log2_warp(vloc, q, P, lane) + VD.slack;
+    if (bnd < 55.f) {
+        venn_warp_terms<uint64_t>(vloc, V, VD, reinterpret_cast<uint64_t*>(rows), lane, acc);
+    } else if (bnd < 119.f) {
+        venn_warp_terms<u128>(vloc, V, VD, rows, lane, acc);
+    } else {
+        for (int pi = lane; pi < P.nprog; pi += 32) {
+            const FringeProg fp = P.prog[pi];
+            bool o = false;
+            const u128 f = fc_dispatch<STACK>(vloc, q, fp, o);
+            acc.add(fp.pat, f, o);
+        }
+    }
 }
 
 // ------------------------------------------------------------------------
@@ -1078,7 +1171,8 @@ __global__ void __launch_bounds__(kTriWarps * 32) tri_core_kernel(GraphDev G, Or
                                                                    const CoreProg P, WorkDesc W,
                                                                    const int* __restrict__ sup, const VennDev VD,
                                                                    const Sink S) {
-    extern __shared__ u128 s_rows[];                 // Venn-table binomial rows [entry][thread]
+    extern __shared__ u128 s_rows[];                     // small tables: rows [entry][thread]
+    __shared__ u128 s_vrows[kTriWarps][kMaxVennRows];   // large tables: rows per warp
     __shared__ uint32_t s_leaf[kTriWarps][64][6];   // u, v, w, e(uv), e(uw), e(vw)
     __shared__ uint32_t s_venn[kTriWarps][64][8];   // Venn over the q anchors
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
@@ -1174,27 +1268,34 @@ __global__ void __launch_bounds__(kTriWarps * 32) tri_core_kernel(GraphDev G, Or
         }
         __syncwarp();
         if (VD.n) {
-            // (2) fc by the Venn term table, one leaf per lane, every program
-            for (int base = 0; base < cnt; base += 32) {
-                const int li = base + lane;
-                const bool mine = li < cnt;
-                uint32_t vloc[8];
-                float bnd = 0.f;
-                if (mine) {
+            if (VD.warp) {   // (2) fc by the Venn term table, one leaf at a time per warp
+                for (int li = 0; li < cnt; ++li) {
+                    uint32_t vloc[8];
                     for (int k = 0; k < V; ++k) vloc[k] = s_venn[wib][li][k];
-                    bnd = venn_bound_log2(vloc, q, P) + VD.slack;
+                    venn_fc_warp<kTriStack>(vloc, q, P, VD, s_vrows[wib], lane, acc);
                 }
-                const bool all64 = __all_sync(FULLMASK, !mine || bnd < 55.f);
-                if (mine && all64) {
-                    venn_terms_eval<uint64_t>(vloc, V, VD, (uint64_t*)(s_rows + threadIdx.x), 2 * blockDim.x, acc);
-                } else if (mine && bnd < 119.f) {
-                    venn_terms_eval<u128>(vloc, V, VD, s_rows + threadIdx.x, blockDim.x, acc);
-                } else if (mine) {                     // checked Listing 5 per program
-                    for (int pi = 0; pi < nprog; ++pi) {
-                        const FringeProg fp = P.prog[pi];
-                        bool o = false;
-                        const u128 f = fc_dispatch<kTriStack>(vloc, q, fp, o);
-                        acc.add(fp.pat, f, o);
+            } else {         // (2) small tables: one leaf per lane, rows per thread
+                for (int base = 0; base < cnt; base += 32) {
+                    const int li = base + lane;
+                    const bool mine = li < cnt;
+                    uint32_t vloc[8];
+                    float bnd = 0.f;
+                    if (mine) {
+                        for (int k = 0; k < V; ++k) vloc[k] = s_venn[wib][li][k];
+                        bnd = venn_bound_log2(vloc, q, P) + VD.slack;
+                    }
+                    const bool all64 = __all_sync(FULLMASK, !mine || bnd < 55.f);
+                    if (mine && all64) {
+                        venn_terms_eval<uint64_t>(vloc, V, VD, (uint64_t*)(s_rows + threadIdx.x), 2 * blockDim.x, acc);
+                    } else if (mine && bnd < 119.f) {
+                        venn_terms_eval<u128>(vloc, V, VD, s_rows + threadIdx.x, blockDim.x, acc);
+                    } else if (mine) {                     // checked Listing 5 per program
+                        for (int pi = 0; pi < nprog; ++pi) {
+                            const FringeProg fp = P.prog[pi];
+                            bool o = false;
+                            const u128 f = fc_dispatch<kTriStack>(vloc, q, fp, o);
+                            acc.add(fp.pat, f, o);
+                        }
                     }
                 }
             }
@@ -1351,6 +1452,7 @@ __global__ void __launch_bounds__(kCoreWarps * 32) core_kernel(GraphDev G, Orien
                                                                 const VennDev VD, const Sink S,
                                                                 unsigned long long* queue) {
     extern __shared__ uint32_t smem[];
+    __shared__ u128 s_vrows[kCoreWarps][kMaxVennRows];   // Venn-table binomial rows, per warp
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     const int q = P.q, V = 1 << q, p = P.p, nprog = P.nprog;
     uint32_t* s_leaf = smem + wib * (32 * FSGC_MAXC);                       // [32][MAXC]
@@ -1505,7 +1607,13 @@ __global__ void __launch_bounds__(kCoreWarps * 32) core_kernel(GraphDev G, Orien
             __syncwarp();
         }
         __syncwarp();
-        if (VD.n) {                               // fc by the Venn term table, leaf per lane
+        if (VD.n && VD.warp) {                    // fc by the Venn term table, leaf by leaf
+            for (int li = 0; li < cnt; ++li) {
+                uint32_t vloc[1 << FSGC_MAXQ];
+                for (int k = 0; k < V; ++k) vloc[k] = s_venn[li * V + k];
+                venn_fc_warp<FSGC_FC_STACK>(vloc, q, P, VD, s_vrows[wib], lane, acc);
+            }
+        } else if (VD.n) {                        // small tables: a leaf per lane
             u128* rows = reinterpret_cast<u128*>(smem + kCoreWarps * 32 * (FSGC_MAXC + V));
             const bool mine = lane < cnt;
             uint32_t vloc[1 << FSGC_MAXQ];
@@ -2158,16 +2266,24 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
             P->terms = T;
         }
         // Venn tables -> passes: rows in dynamic shared memory, grids re-sized
-        const size_t kStatic = 40 * 1024;    // the kernels' static shared memory (upper bound)
         for (size_t i = 0; i < P->passes.size(); ++i) {
             PassExec& X = P->passes[i];
             X.vd = P->terms->vhdr[i];
             if (!X.vd.n) continue;
+            // small tables: a diagram per lane, rows per thread in dynamic
+            // shared memory; large ones (more than 48 KB of rows per block or
+            // FSGC_VENN_WARP_TERMS terms): a diagram per warp, rows per warp
             const int threads = X.kind == 3 ? kTriWarps * 32 : kCoreWarps * 32;
-            X.smem_vd = (size_t)X.vd.nrows * sizeof(u128) * threads;
-            if (X.smem_vd + X.smem + kStatic > 227 * 1024) { X.vd.n = 0; X.smem_vd = 0; continue; }
-            const int64_t per = (int64_t)nsm * occupancy(kernel_for(X.kind, X.npc), threads, X.smem + X.smem_vd);
-            X.grid = std::max<int64_t>(1, std::min<int64_t>(X.grid, per));
+            const size_t lane_rows = (size_t)X.vd.nrows * sizeof(u128) * threads;
+            X.vd.warp = (lane_rows > 48 * 1024 || X.vd.n >= tune("FSGC_VENN_WARP_TERMS", 1024)) ? 1 : 0;
+            X.smem_vd = X.vd.warp ? 0 : lane_rows;
+            if (!X.vd.warp) {
+                const int64_t per = (int64_t)nsm * occupancy(kernel_for(X.kind, X.npc), threads, X.smem + X.smem_vd);
+                X.grid = std::max<int64_t>(1, std::min<int64_t>(X.grid, per));
+            }
+            if (tune("FSGC_VENN_INFO", 0))
+                fprintf(stderr, "[venn] pass kind %d: %d terms, %d rows, %s mode\n", X.kind, X.vd.n, X.vd.nrows,
+                        X.vd.warp ? "warp" : "lane");
         }
     }
     P->ev.resize(2 + 2 * P->passes.size());

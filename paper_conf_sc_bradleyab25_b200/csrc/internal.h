@@ -79,7 +79,7 @@ struct fsgc_pattern {
 // Limits of one count pass (one core-isomorphism class of patterns).
 #define FSGC_MAXC FSGC_MAX_CORE
 #define FSGC_MAXQ FSGC_MAX_VENN_BITS
-#define FSGC_MAXPROG 48
+#define FSGC_MAXPROG 192
 #define FSGC_MAXT 16
 #define FSGC_MAXPATS FSGC_MAX_BATCH
 #define FSGC_FC_STACK 64
