@@ -313,7 +313,9 @@ def combine_partials(part: Sequence[CountResult], group=None, device=None) -> Li
         cnt = None if flags[k] else fsgc_finalize(raws[k], r.divisor, False)
         out.append(CountResult(count=cnt, raw=raws[k], divisor=r.divisor,
                                core_matches=h[5 * len(part) + k], overflow=flags[k],
-                               root_pattern_vertex=r.root_pattern_vertex))
+                               root_pattern_vertex=r.root_pattern_vertex, kernel_ms=r.kernel_ms,
+                               aux_ms=r.aux_ms, kernel_launches=r.kernel_launches,
+                               pass_index=r.pass_index, pass_kind=r.pass_kind))
     return out
 
 

@@ -2183,15 +2183,21 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
         }
         X.uses_sup = X.kind != 0 && g->m > 0;
         if (X.uses_sup && P->sup_first < 0) P->sup_first = (int)P->passes.size();
-        X.parts_off = kHdrBytes;
-        X.bytes = (X.parts_off + (size_t)X.grid * sizeof(BlockPartial) + 255) & ~(size_t)255;
-        X.ws_off = off;
-        off += X.bytes;
+        X.bytes = ((size_t)X.grid * sizeof(BlockPartial) + 255) & ~(size_t)255;   // block partials
         P->passes.push_back(X);
     }
+    // workspace: [pass headers][support queue counters (256 B)][support
+    // array][pass block partials] -- the zeroed part is one contiguous range
+    const size_t np_ = P->passes.size();
+    P->sup_off = np_ * kHdrBytes + 256;
+    off = P->sup_off + (P->sup_first >= 0 ? (((size_t)g->m * sizeof(int) + 255) & ~(size_t)255) : 0);
+    for (size_t i = 0; i < np_; ++i) {
+        PassExec& X = P->passes[i];
+        X.ws_off = i * kHdrBytes;
+        X.parts_off = off - X.ws_off;
+        off += X.bytes;
+    }
     if (P->sup_first >= 0) {
-        P->sup_off = off + 256;
-        off += 256 + (((size_t)g->m * sizeof(int) + 255) & ~(size_t)255);
         P->grid_sup = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy((const void*)support_kernel, 256, 0),
                                                              (g->nsup_heavy + 255) / 256));
         typedef SupLayout<FSGC_SUP_CAPW> LS;
@@ -2323,9 +2329,18 @@ extern "C" int fsgc_plan_enqueue_stage(const fsgc_plan* P, void* workspace, void
     GraphDev G{g->offsets, g->adj, g->row, g->osrc, g->odst};
     OrientDev O{g->split, g->oofs};
     int* dsup = (int*)((unsigned char*)workspace + P->sup_off);
+    const size_t np_ = P->passes.size();
+    const size_t sup_bytes = P->sup_first >= 0 ? (size_t)g->m * sizeof(int) : 0;
+    // zero the headers (count stage) and the queue + support array (support
+    // stage): one memset when both stages run
+    if ((stages & FSGC_STAGE_ALL) == FSGC_STAGE_ALL)
+        FSGC_CUDA(cudaMemsetAsync(workspace, 0, P->sup_off + sup_bytes, st));
+    else if (stages & FSGC_STAGE_COUNT)
+        FSGC_CUDA(cudaMemsetAsync(workspace, 0, np_ * kHdrBytes, st));
+    else
+        FSGC_CUDA(cudaMemsetAsync((unsigned char*)workspace + np_ * kHdrBytes, 0, 256 + sup_bytes, st));
     if ((stages & FSGC_STAGE_SUPPORT) && P->sup_first >= 0) {   // (A) per-edge common-neighbour counts
         unsigned long long* dq = (unsigned long long*)((unsigned char*)dsup - 256);   // 2 queue counters
-        FSGC_CUDA(cudaMemsetAsync(dq, 0, 256 + (size_t)g->m * sizeof(int), st));
         FSGC_CUDA(cudaEventRecordWithFlags(P->ev[0], st, evflags));
         // FSGC_SUP_MERGE_ONLY=1 (experiments): the merge kernel over every
         // oriented edge (the work list holds the light ones after the heavy)
@@ -2359,7 +2374,6 @@ extern "C" int fsgc_plan_enqueue_stage(const fsgc_plan* P, void* workspace, void
     for (size_t pi = 0; pi < P->passes.size(); ++pi) {
         const PassExec& X = P->passes[pi];
         unsigned char* base = (unsigned char*)workspace + X.ws_off;
-        FSGC_CUDA(cudaMemsetAsync(base, 0, kHdrBytes, st));
         AccDev* dacc = (AccDev*)base;
         unsigned long long* dmatch = (unsigned long long*)(base + sizeof(AccDev) * FSGC_MAXPATS);
         unsigned long long* dqueue = dmatch + 1;
@@ -2389,9 +2403,10 @@ extern "C" int fsgc_plan_enqueue_stage(const fsgc_plan* P, void* workspace, void
                                            X.smem + X.smem_vd, st));
         }
         FSGC_CUDA(cudaEventRecordWithFlags(P->ev[3 + 2 * pi], st, evflags));
-        FSGC_CUDA(cudaMemcpyAsync((unsigned char*)raw_out + pi * kRawPassBytes, base, kRawPassBytes - 8,
-                                  cudaMemcpyDefault, st));
     }
+    // every pass's raw sums in one strided copy (header pitch -> raw pitch)
+    FSGC_CUDA(cudaMemcpy2DAsync(raw_out, kRawPassBytes, workspace, kHdrBytes, kRawPassBytes - 8, np_,
+                                cudaMemcpyDefault, st));
     return FSGC_OK;
 }
 

@@ -31,14 +31,24 @@ METRICS = [
 
 
 def short(name):
-    for k in ("support_kernel", "edge_fc_kernel", "core_kernel", "vertex_core_kernel", "tri_core_kernel"):
+    import re
+    m = re.search(r"support_hash_kernel<\d+>", name)
+    if m:
+        return m.group(0)
+    for k in ("support_kernel", "edge_fc_kernel", "tri_core_kernel", "vertex_core_kernel", "core_kernel"):
         if k in name:
             return k
     return name.split("(")[0][-40:]
 
 
 def raw_page(rep):
-    out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    """rows of the raw page: from an .ncu-rep (via ncu -i) or from its
+    exported CSV (ncu -i REP --page raw --csv > X_raw.csv, done on the GPU box
+    so the large report need not travel back)"""
+    if rep.endswith(".csv"):
+        out = open(rep).read()
+    else:
+        out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(out)))
     hdr, units = rows[0], rows[1]
     res = []
@@ -84,6 +94,8 @@ def main():
     ap.add_argument("--launches")
     a = ap.parse_args()
     rep = a.rep or os.path.join(ROOT, "gpurun_out", f"prof_{a.tag}_{a.workload}.ncu-rep")
+    if not os.path.exists(rep) and os.path.exists(rep.replace(".ncu-rep", "_raw.csv")):
+        rep = rep.replace(".ncu-rep", "_raw.csv")
     lpath = a.launches or os.path.join(ROOT, "gpurun_out", f"launches_{a.tag}_{a.workload}.csv")
     md = [f"# ncu summary {a.tag} / {a.workload}", ""]
     kern = {}
@@ -100,6 +112,18 @@ def main():
             kern[k]["dram_bytes_per_launch"] = (rd or 0) + (wr or 0)
         md.append("")
         md.append("(units as ncu prints them in the raw page; `dram__bytes_*` are per launch)")
+        md += ["", "### warp stall reasons (PC sampling, top 6 per kernel)", ""]
+        for d in raw_page(rep):
+            st = []
+            for h, v in d.items():
+                if h.startswith("smsp__pcsamp_warps_issue_stalled_") and not h.endswith("not_issued"):
+                    x = num(v)
+                    if x:
+                        st.append((x, h.replace("smsp__pcsamp_warps_issue_stalled_", "")))
+            st.sort(reverse=True)
+            tot = sum(x for x, _ in st) or 1.0
+            md.append(f"- {short(d.get('Kernel Name', '?'))}: " +
+                      ", ".join(f"{h} {100 * x / tot:.0f}%" for x, h in st[:6]))
     if os.path.exists(lpath):
         agg = launches(lpath)
         tot = sum(sum(v) for v in agg.values())

@@ -311,13 +311,16 @@ def test_edge_core_counts_beyond_64_bits():
         assert not r.overflow and r.count == oracle.fringe_count(gadj, P.n, P.edges, P.core), P.name
 
 
-def test_sharded_support_stages_sum_to_whole():
+@pytest.mark.parametrize("algo", ["merge", "wedge-hash"])
+def test_sharded_support_stages_sum_to_whole(algo, monkeypatch):
     """FSGC_FLAG_SHARD_SUPPORT: each shard lists its interleaved part of the
     triangles into a partial support array; the SUM of the partial arrays
     (what the multi-GPU all-reduce computes) is the full support array, and
     stage 2 on it gives per-shard raws that sum to the unsharded raw -- for
-    an edge-core, a triangle-core and a general-core pass in one plan."""
+    an edge-core, a triangle-core and a general-core pass in one plan, with
+    either support algorithm (the hash kernels deal their units)."""
     from paper_conf_sc_bradleyab25_b200 import _lib
+    monkeypatch.setenv("FSGC_SUP_HASH_MIN_M", "0" if algo == "wedge-hash" else str(1 << 40))
     n, e, _ = workload("pl2k")
     g = F.fsgc_load_graph(e, n)
     pats = [F.compile_named(PATTERNS[x]) for x in ["2-tailed-triangle", "tricore+3f", "k4core+2f", "cycle4"]]
