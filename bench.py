@@ -239,10 +239,17 @@ def main():
     import numpy as np
     import torch
     import torch.distributed as dist
+    # FSGC_BENCH_BACKEND=gloo (testing the N>1 path on a 1-GPU box: ranks
+    # share the visible GPUs round-robin); the product path is NCCL
+    backend = os.environ.get("FSGC_BENCH_BACKEND", "nccl")
+    local = local % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", rank=rank, world_size=world, device_id=dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", rank=rank, world_size=world, device_id=dev)
+        else:
+            dist.init_process_group(backend, rank=rank, world_size=world)
     import paper_conf_sc_bradleyab25_b200 as F
 
     n, e, pats = load_workload(args.workload, dev)
