@@ -481,10 +481,12 @@ __global__ void __launch_bounds__(256) support_kernel(GraphDev G, OrientDev O, i
 // <= CAP: long tails, streamed one at a time, sup_slice_stream).  One warp
 // per unit, its own table sized to out(b) (load factor <= 1/2), no block
 // barriers.
-template <int CAPT>
+// FSGC_SUP_BIG (experiments) picks the large-table variant: 0 streamed
+// tails, 4 warps; 1 concatenated tails (sup_slice), 4 warps; 2 streamed, 2 warps
+template <int CAPT, bool STR = (CAPT > FSGC_SUP_CAPW), int NW = (STR ? 4 : 8)>
 struct SupLayout {
-    static constexpr bool STREAM = CAPT > FSGC_SUP_CAPW;
-    static constexpr int WARPS = STREAM ? 4 : 8;
+    static constexpr bool STREAM = STR;
+    static constexpr int WARPS = NW;
     static constexpr int HS = 2 * CAPT;
     static constexpr size_t table_bytes = (size_t)HS * 4 + (size_t)HS * 2 + (size_t)CAPT * 4;
     static constexpr size_t slice_bytes = STREAM ? 0 : (size_t)(FSGC_SUP_SEG + 4) * 4 + (size_t)4 * FSGC_SUP_SEG * 4;
@@ -633,11 +635,11 @@ __device__ __forceinline__ void sup_slice_stream(const GraphDev& G, const Orient
     }
 }
 
-template <int CAPT>
-__global__ void __launch_bounds__(SupLayout<CAPT>::WARPS * 32, 1) support_hash_kernel(
+template <int CAPT, bool STR = (CAPT > FSGC_SUP_CAPW), int NW = (STR ? 4 : 8)>
+__global__ void __launch_bounds__(NW * 32, 1) support_hash_kernel(
     GraphDev G, OrientDev O, const int32_t* __restrict__ rev, const uint64_t* __restrict__ units, int64_t nunits,
     int* __restrict__ sup, unsigned long long* queue, int shard, int nshards) {
-    typedef SupLayout<CAPT> Lay;
+    typedef SupLayout<CAPT, STR, NW> Lay;
     extern __shared__ __align__(16) unsigned char s_sup[];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     unsigned char* tb = s_sup + w * Lay::warp_bytes;
@@ -1769,6 +1771,28 @@ int tune(const char* name, int dflt) {
     return r;
 }
 
+// the large-table support kernel (FSGC_SUP_BIG variant, see SupLayout), its
+// warps per block and dynamic shared memory
+const void* big_support_kernel(int* warps, size_t* bytes) {
+    const int mode = tune("FSGC_SUP_BIG", 0);
+    if (mode == 1) {
+        typedef SupLayout<FSGC_SUP_CAP, false, 4> L;
+        *warps = L::WARPS;
+        if (bytes) *bytes = L::bytes;
+        return (const void*)support_hash_kernel<FSGC_SUP_CAP, false, 4>;
+    }
+    if (mode == 2) {
+        typedef SupLayout<FSGC_SUP_CAP, true, 2> L;
+        *warps = L::WARPS;
+        if (bytes) *bytes = L::bytes;
+        return (const void*)support_hash_kernel<FSGC_SUP_CAP, true, 2>;
+    }
+    typedef SupLayout<FSGC_SUP_CAP> L;
+    *warps = L::WARPS;
+    if (bytes) *bytes = L::bytes;
+    return (const void*)support_hash_kernel<FSGC_SUP_CAP>;
+}
+
 // resident blocks per SM of a kernel (cached per function / block / smem)
 int occupancy(const void* fn, int threads, size_t smem) {
     static std::mutex mu;
@@ -2201,13 +2225,16 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
         P->grid_sup = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy((const void*)support_kernel, 256, 0),
                                                              (g->nsup_heavy + 255) / 256));
         typedef SupLayout<FSGC_SUP_CAPW> LS;
-        typedef SupLayout<FSGC_SUP_CAP> LB;
         P->grid_hash = std::max<int64_t>(1, std::min<int64_t>(
             (int64_t)nsm * occupancy((const void*)support_hash_kernel<FSGC_SUP_CAPW>, LS::WARPS * 32, LS::bytes),
             (g->nsup_units + LS::WARPS - 1) / LS::WARPS));
+        int warps_big = 0;
+        const void* fn_big = big_support_kernel(&warps_big, nullptr);
+        size_t bytes_big = 0;
+        big_support_kernel(&warps_big, &bytes_big);
         P->grid_hash_big = std::max<int64_t>(1, std::min<int64_t>(
-            (int64_t)nsm * occupancy((const void*)support_hash_kernel<FSGC_SUP_CAP>, LB::WARPS * 32, LB::bytes),
-            (g->nsup_units_big + LB::WARPS - 1) / LB::WARPS));
+            (int64_t)nsm * occupancy(fn_big, warps_big * 32, bytes_big),
+            (g->nsup_units_big + warps_big - 1) / warps_big));
         if ((opts.flags & FSGC_FLAG_SHARD_SUPPORT) && opts.shard_count > 1) {
             P->sup_shard = opts.shard_index;
             P->sup_nshards = opts.shard_count;
@@ -2341,15 +2368,18 @@ extern "C" int fsgc_plan_enqueue_stage(const fsgc_plan* P, void* workspace, void
         FSGC_CUDA(cudaMemsetAsync((unsigned char*)workspace + np_ * kHdrBytes, 0, 256 + sup_bytes, st));
     if ((stages & FSGC_STAGE_SUPPORT) && P->sup_first >= 0) {   // (A) per-edge common-neighbour counts
         unsigned long long* dq = (unsigned long long*)((unsigned char*)dsup - 256);   // 2 queue counters
+        unsigned long long* dq1 = dq + 1;
         FSGC_CUDA(cudaEventRecordWithFlags(P->ev[0], st, evflags));
         // FSGC_SUP_MERGE_ONLY=1 (experiments): the merge kernel over every
         // oriented edge (the work list holds the light ones after the heavy)
         const bool merge_only = tune("FSGC_SUP_MERGE_ONLY", 0) != 0;
         if (g->nsup_units_big > 0 && !merge_only) {
-            typedef SupLayout<FSGC_SUP_CAP> LB;
-            support_hash_kernel<FSGC_SUP_CAP><<<(int)P->grid_hash_big, LB::WARPS * 32, LB::bytes, st>>>(
-                G, O, g->rev, g->sup_units_big, g->nsup_units_big, dsup, dq + 1, P->sup_shard, P->sup_nshards);
-            FSGC_CUDA(cudaGetLastError());
+            int nw = 0;
+            size_t nb = 0;
+            const void* fn = big_support_kernel(&nw, &nb);
+            void* args[] = {(void*)&G, (void*)&O, (void*)&g->rev, (void*)&g->sup_units_big, (void*)&g->nsup_units_big,
+                            (void*)&dsup, (void*)&dq1, (void*)&P->sup_shard, (void*)&P->sup_nshards};
+            FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)P->grid_hash_big), dim3(nw * 32), args, nb, st));
         }
         if (g->nsup_units > 0 && !merge_only) {
             typedef SupLayout<FSGC_SUP_CAPW> LS;
