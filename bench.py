@@ -50,7 +50,8 @@ WORKLOAD_DESC = {
     "rmat16": "4-clique cores with 1-6 and a diamond core with 1 mixed fringe on RMAT scale 16 "
               "(configs[2] patterns; Table 1's rmat16.sym scale)",
     "pl10m": "Fig. 4 16-vertex/25-edge pattern on synthetic power-law graph, 10M edges (configs[3])",
-    "rmat26": "triangle and 4-cycle cores with fringes on RMAT scale 26 (configs[4])",
+    "rmat26": "triangle and k-tailed triangles (k=1..4) on RMAT scale 26, 1.07B raw / 1.05B "
+              "distinct edges (configs[4] graph; patterns decomposed to the edge core)",
 }
 
 

@@ -145,7 +145,11 @@ CONFIG_PATTERNS = {
     "rmat22": ["triangle", "diamond"] + [f"{k}-tailed-triangle" for k in range(1, 5)],
     "rmat16": [f"k4core+{f}f" for f in range(1, 7)] + ["diamondcore+1f"],
     "pl10m": ["fig4"],
-    "rmat26": [f"tricore+{f}f" for f in range(1, 7)] + [f"c4core+{f}f" for f in range(1, 7)],
+    # configs[4]: triangle-with-fringes patterns on RMAT-26 as the compiler
+    # decomposes them (edge core, R13); the forced triangle / 4-cycle
+    # core sets below do not finish a step at this scale (Next)
+    "rmat26": ["triangle"] + [f"{k}-tailed-triangle" for k in range(1, 5)],
+    "rmat26-forced-cores": [f"tricore+{f}f" for f in range(1, 7)] + [f"c4core+{f}f" for f in range(1, 7)],
 }
 
 

@@ -1191,6 +1191,17 @@ __global__ void __launch_bounds__(kTriWarps * 32) tri_core_kernel(GraphDev G, Or
             if ((F >> P.anchor_pos[b]) & 1) M |= 1 << b;
         proj[F] = M;
     }
+    // t enters region F with sign +1 (|F| odd) or -1 (|F| = 2); the Venn over
+    // the anchors needs t only if some anchor region collects a nonzero sum of
+    // those signs (only when all three core vertices are anchors)
+    bool need_t = false;
+    {
+        int tco[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+#pragma unroll
+        for (int F = 1; F < 8; ++F) tco[proj[F]] += (__popc(F) & 1) ? 1 : -1;
+#pragma unroll
+        for (int M = 1; M < 8; ++M) need_t |= tco[M] != 0;
+    }
     // this shard's roots, transposed over the grid (see edge_fc_kernel)
     const int64_t total = W.end - W.begin;
     const int64_t nchunks = (total + 31) / 32;
@@ -1223,8 +1234,8 @@ __global__ void __launch_bounds__(kTriWarps * 32) tri_core_kernel(GraphDev G, Or
                 dv = (int)(__ldg(G.offs + lv + 1) - __ldg(G.offs + lv));
                 dw = (int)(__ldg(G.offs + lw + 1) - __ldg(G.offs + lw));
             }
-            const bool heavy = mine && du > kTriLight;
-            if (mine && !heavy) {
+            const bool heavy = mine && need_t && du > kTriLight;
+            if (mine && need_t && !heavy) {
                 Cursor cv, cw;
                 cv.init(G, H, lv);
                 cw.init(G, H, lw);

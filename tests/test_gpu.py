@@ -3,6 +3,7 @@ against the oracle on the same seeded inputs.  Integer results: bit-exact.
 
 Expected values come only from ``oracle/`` (or the paper, for Fig. 2).
 """
+import os
 import random
 from math import comb
 
@@ -463,3 +464,30 @@ def test_wedge_hash_support_equals_merge(wl, monkeypatch):
         out.append((plan.support().clone(), [r.raw for r in plan.decode()]))
     assert torch.equal(out[0][0], out[1][0])
     assert out[0][1] == out[1][1]
+
+
+def _one_count_subprocess(wl, names, env_extra):
+    """counts of ``names`` on workload ``wl`` in a fresh process (the library
+    reads its FSGC_* knobs once per process)"""
+    import ast
+    import subprocess
+    import sys
+    env = dict(os.environ, **env_extra)
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    out = subprocess.run([sys.executable, os.path.join(root, "scripts", "one_count.py"), wl, ",".join(names), "1"],
+                         env=env, capture_output=True, text=True, timeout=600, check=True).stdout
+    d = ast.literal_eval(out.strip().splitlines()[-1])
+    return {k: v[0] for k, v in d.items()}
+
+
+def test_rmat26_full_size_wedge_hash_equals_merge():
+    """configs[4] graph at full size (RMAT-26, 1.05e9 distinct edges): the
+    triangle and k-tailed-triangle counts of the bench path (wedge-hash
+    support pass) equal those of the independent merge-only support pass
+    (FSGC_SUP_MERGE_ONLY=1), and the triangle count is below the Turan-type
+    bound m^1.5 (property checks at a size the oracle cannot reach)."""
+    names = ["triangle", "1-tailed-triangle", "2-tailed-triangle"]
+    a = _one_count_subprocess("rmat26", names, {})
+    b = _one_count_subprocess("rmat26", names, {"FSGC_SUP_MERGE_ONLY": "1"})
+    assert a == b, (a, b)
+    assert 0 < a["triangle"] < (1_051_923_859 ** 1.5)
