@@ -1344,7 +1344,10 @@ __global__ void __launch_bounds__(kTriWarps * 32) tri_core_kernel(GraphDev G, Or
             const int64_t ou = __ldg(G.offs + u), ou1 = __ldg(G.offs + u + 1);
             const int64_t ov = __ldg(G.offs + v), ov1 = __ldg(G.offs + v + 1);
             if (W.degfilter && ((int)(ou1 - ou) < P.mindeg[0] || (int)(ov1 - ov) < P.mindeg[1])) continue;
-            su = __ldg(O.split + u); pa = su; ea = ou1;
+            if (__ldg(sup + e) == 0) continue;       // no triangle on (u, v) at all
+            // w > v: the merge starts in N+(u) right after v (v's position
+            // in N+(u) is e's oriented offset)
+            su = __ldg(O.split + u); pa = su + (e - __ldg(O.oofs + u)) + 1; ea = ou1;
             sv = __ldg(O.split + v); pb = sv; eb = ov1;
             have = true;
         }
