@@ -1787,7 +1787,19 @@ int tune(const char* name, int dflt) {
 
 // the large-table support kernel (FSGC_SUP_BIG variant, see SupLayout), its
 // warps per block and dynamic shared memory
-const void* big_support_kernel(int* warps, size_t* bytes) {
+const void* big_support_kernel(int* warps, size_t* bytes, int cap) {
+    if (cap == 4096) {
+        typedef SupLayout<4096, true, 1> L;
+        *warps = L::WARPS;
+        if (bytes) *bytes = L::bytes;
+        return (const void*)support_hash_kernel<4096, true, 1>;
+    }
+    if (cap == 2048) {
+        typedef SupLayout<2048, true, 2> L;
+        *warps = L::WARPS;
+        if (bytes) *bytes = L::bytes;
+        return (const void*)support_hash_kernel<2048, true, 2>;
+    }
     const int mode = tune("FSGC_SUP_BIG", 0);
     if (mode == 1) {
         typedef SupLayout<FSGC_SUP_CAP, false, 4> L;
@@ -2243,9 +2255,9 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
             (int64_t)nsm * occupancy((const void*)support_hash_kernel<FSGC_SUP_CAPW>, LS::WARPS * 32, LS::bytes),
             (g->nsup_units + LS::WARPS - 1) / LS::WARPS));
         int warps_big = 0;
-        const void* fn_big = big_support_kernel(&warps_big, nullptr);
+        const void* fn_big = big_support_kernel(&warps_big, nullptr, g->sup_cap_big);
         size_t bytes_big = 0;
-        big_support_kernel(&warps_big, &bytes_big);
+        big_support_kernel(&warps_big, &bytes_big, g->sup_cap_big);
         P->grid_hash_big = std::max<int64_t>(1, std::min<int64_t>(
             (int64_t)nsm * occupancy(fn_big, warps_big * 32, bytes_big),
             (g->nsup_units_big + warps_big - 1) / warps_big));
@@ -2390,7 +2402,7 @@ extern "C" int fsgc_plan_enqueue_stage(const fsgc_plan* P, void* workspace, void
         if (g->nsup_units_big > 0 && !merge_only) {
             int nw = 0;
             size_t nb = 0;
-            const void* fn = big_support_kernel(&nw, &nb);
+            const void* fn = big_support_kernel(&nw, &nb, g->sup_cap_big);
             void* args[] = {(void*)&G, (void*)&O, (void*)&g->rev, (void*)&g->sup_units_big, (void*)&g->nsup_units_big,
                             (void*)&dsup, (void*)&dq1, (void*)&P->sup_shard, (void*)&P->sup_nshards};
             FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)P->grid_hash_big), dim3(nw * 32), args, nb, st));

@@ -182,14 +182,14 @@ __global__ void rev_keys(const int32_t* __restrict__ osrc, const int32_t* __rest
 // small-table units ceil(in(b) / SEG) when 1 <= out(b) <= CAPW, large-table
 // units ceil(in(b) / SEG) when CAPW < out(b) <= CAP
 __global__ void unit_counts(const int64_t* __restrict__ offs, const int64_t* __restrict__ split, int64_t n,
-                            int64_t* __restrict__ cnt, int64_t* __restrict__ cnt_big) {
+                            int64_t* __restrict__ cnt, int64_t* __restrict__ cnt_big, int64_t cap) {
     for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b <= n;
          b += (int64_t)gridDim.x * blockDim.x) {
         int64_t c = 0, cb = 0;
         if (b < n) {
             const int64_t in = split[b] - offs[b], out = offs[b + 1] - split[b];
             if (in >= 1 && out >= 1 && out <= FSGC_SUP_CAPW) c = (in + FSGC_SUP_SEG - 1) / FSGC_SUP_SEG;
-            if (in >= 1 && out > FSGC_SUP_CAPW && out <= FSGC_SUP_CAP) cb = (in + FSGC_SUP_SEG - 1) / FSGC_SUP_SEG;
+            if (in >= 1 && out > FSGC_SUP_CAPW && out <= cap) cb = (in + FSGC_SUP_SEG - 1) / FSGC_SUP_SEG;
         }
         cnt[b] = c;
         cnt_big[b] = cb;
@@ -420,6 +420,12 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
     int64_t hash_min_m = 1 << 20;
     if (const char* v = getenv("FSGC_SUP_HASH_MIN_M")) hash_min_m = atoll(v);
     const bool use_hash = m >= hash_min_m;
+    // FSGC_SUP_CAP_BIG (experiments): large-table cap 1024 (default), 2048 or 4096
+    int64_t cap_big = FSGC_SUP_CAP;
+    if (const char* v = getenv("FSGC_SUP_CAP_BIG")) {
+        const int64_t c = atoll(v);
+        if (c == 2048 || c == 4096) cap_big = c;
+    }
     if (m > 0 && use_hash) {
         {   // rev = oriented edge ids in (b, a) order = the in-entries' CSR order
             DevBuf<uint64_t> rk0, rk1;
@@ -440,7 +446,7 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
         }
         FSGC_CUDA(ucnt.alloc(n + 1, st));
         FSGC_CUDA(ucnt_big.alloc(n + 1, st));
-        unit_counts<<<grid_for(n + 1), 256, 0, st>>>(offs.ptr, split.ptr, n, ucnt.ptr, ucnt_big.ptr);
+        unit_counts<<<grid_for(n + 1), 256, 0, st>>>(offs.ptr, split.ptr, n, ucnt.ptr, ucnt_big.ptr, cap_big);
         FSGC_CUDA(cudaGetLastError());
         size_t b = 0;
         FSGC_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, b, ucnt.ptr, ucnt.ptr, n + 1, st));
@@ -463,7 +469,7 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
         FSGC_CUDA(i1.alloc(m, st));
         support_work_keys<<<grid_for(m), 256, 0, st>>>(offs.ptr, split.ptr, osrc.ptr, odst.ptr, m, k0.ptr, sorder.ptr,
                                                        (unsigned long long*)dnum.ptr,
-                                                       use_hash ? (int64_t)FSGC_SUP_CAP : (int64_t)-1);
+                                                       use_hash ? cap_big : (int64_t)-1);
         FSGC_CUDA(cudaGetLastError());
         cub::DoubleBuffer<uint32_t> dk(k0.ptr, k1.ptr);
         cub::DoubleBuffer<int32_t> dv(sorder.ptr, i1.ptr);
@@ -547,6 +553,7 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
     g->nsup_units = nunits;
     g->sup_units_big = units_big.take();
     g->nsup_units_big = nunits_big;
+    g->sup_cap_big = (int32_t)cap_big;
     g->rev = rev.take();
     g->hub_base = hub_base;
     g->hub_words = hub_words;

@@ -45,6 +45,7 @@ struct fsgc_graph {
     int64_t nsup_units = 0;
     uint64_t* sup_units_big = nullptr;   // [nsup_units_big]
     int64_t nsup_units_big = 0;
+    int32_t sup_cap_big = FSGC_SUP_CAP;   // max out(b) of a large-table middle (FSGC_SUP_CAP_BIG)
     // rev[i - oofs[b]] = oriented index of (a, b) for the in-entry a = adj[i]
     // of row b (i in [offs[b], split[b])) -- the position of b in N+(a)
     int32_t* rev = nullptr;          // [m]
