@@ -80,9 +80,13 @@ typedef struct { uint64_t lo, hi; } fsgc_u128;
  *                   Vertex ids are RELABELED: new id = rank of the vertex in
  *                   (degree ascending, original id ascending) order;
  *                   adjacency lists sorted ascending by new id.
+ * Limits: n < 2^31 and, after deduplication, m < 2^31 undirected edges
+ * (edge ids and CSR positions of the counting kernels are 32-bit: 2m must
+ * fit an unsigned 32-bit index).  RMAT scale 26 (m = 1.05e9) fits.
  * Errors: FSGC_ERR_INVALID for null pointers, bad index_bytes, n <= 0 or
- * n >= 2^31, or an id outside [0, n) (detected on the device); FSGC_ERR_OOM;
- * FSGC_ERR_CUDA.  Synchronises `stream`.
+ * n >= 2^31, m >= 2^31 after deduplication, or an id outside [0, n)
+ * (detected on the device); FSGC_ERR_OOM; FSGC_ERR_CUDA.  Synchronises
+ * `stream`.
  */
 int fsgc_load_graph(const void* edges, int64_t num_input_edges, int index_bytes,
                     int64_t num_vertices, int edges_on_device, void* stream,

@@ -19,6 +19,11 @@ Modules
            fringe counting function fc (Listing 5), scaled by the fringe
            multiplicities and divided by |Aut(P)|.
 
+  cfast    mode 2 with the per-core-map work (Venn by explicit marking,
+           Listing 5) in plain C (oracle/c/core_fringe.c, gcc -fopenmp):
+           the same definition, fast enough for RMAT graphs with hubs;
+           pinned to the Python oracle and to closed forms.
+
 Pins (tests/test_oracle.py, ``-m "not gpu"``): Fig. 2 facts, closed forms
 (k-stars, wedges, trace(A^3)/6, trace(A^4) 4-cycles, tailed triangles), Sec. 3.1
 explicit edge-core formulas, definition-level brute force of fc on explicit

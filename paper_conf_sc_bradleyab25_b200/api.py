@@ -43,6 +43,7 @@ class Graph:
         self.n = info.num_vertices
         self.m = info.num_edges
         self.max_degree = info.max_degree
+        self._plans = {}          # distributed plans of this graph (freed with it)
 
     @property
     def handle(self):
@@ -57,6 +58,9 @@ class Graph:
         return offs, adj[:2 * self.m], order
 
     def free(self):
+        for plan in getattr(self, "_plans", {}).values():
+            plan.free()
+        self._plans = {}
         if self._h:
             lib.fsgc_free_graph(self._h)
             self._h = C.c_void_p(0)
@@ -319,20 +323,19 @@ def combine_partials(part: Sequence[CountResult], group=None, device=None) -> Li
     return out
 
 
-_dist_plans = {}
-
-
 def distributed_plan(graph: Graph, patterns: Sequence[Pattern], rank: int, world: int, **kw) -> Plan:
     """cached plan of this rank's shard: root chunks AND the support pass's
-    chunks dealt round-robin (FSGC_FLAG_SHARD_SUPPORT)"""
-    key = (graph.handle.value, tuple(p.handle.value for p in patterns), rank, world,
-           tuple(sorted(kw.items())))
-    plan = _dist_plans.get(key)
-    if plan is None or plan.graph is not graph:
-        if len(_dist_plans) > 64:
-            _dist_plans.clear()
+    chunks dealt round-robin (FSGC_FLAG_SHARD_SUPPORT).  The cache lives on
+    the graph object and is released by ``Graph.free()``."""
+    key = (tuple(p.handle.value for p in patterns), rank, world, tuple(sorted(kw.items())))
+    plan = graph._plans.get(key)
+    if plan is None:
+        if len(graph._plans) >= 16:
+            for old in graph._plans.values():
+                old.free()
+            graph._plans.clear()
         plan = Plan(graph, patterns, shard_index=rank, shard_count=world, shard_support=world > 1, **kw)
-        _dist_plans[key] = plan
+        graph._plans[key] = plan
     return plan
 
 

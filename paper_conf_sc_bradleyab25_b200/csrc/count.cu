@@ -1422,43 +1422,44 @@ __device__ __forceinline__ int64_t edge_index(const GraphDev& G, const OrientDev
     return __ldg(O.oofs + lo) + (l - __ldg(O.split + lo));
 }
 
-// partition-lattice fc: Z[A] = sum_{e >= A} venn[e]; fc = sum coef prod Z[mask]
-__device__ __noinline__ u128 fc_partition(const uint32_t* venn, int q, const PartTerm* __restrict__ T, int nt,
-                                          bool& ovf) {
+// partition-lattice fc: Z[A] = sum_{e >= A} venn[e]; fc = sum coef prod Z[mask].
+// Exact when every product and partial sum stays below 2^126 in magnitude,
+// which the rising-factorial bound (N + s)^s <= 2^126 guarantees (N = Z[0]);
+// returns false when the bound does not hold -- the caller then evaluates the
+// program by checked Listing 5 instead (exact or flagged, never a
+// conservative overflow)
+__device__ __noinline__ bool fc_partition(const uint32_t* venn, int q, const PartTerm* __restrict__ T, int nt,
+                                          u128& out) {
     int64_t Z[64];
     const int V = 1 << q;
     for (int A = 0; A < V; ++A) Z[A] = A ? venn[A] : 0;
     for (int bb = 0; bb < q; ++bb)
         for (int A = 0; A < V; ++A)
             if (!(A >> bb & 1)) Z[A] += Z[A | (1 << bb)];
-    // 64-bit when the rising-factorial bound (N + s)^s < 2^62 holds, else 128
     uint64_t N = (uint64_t)Z[0];
     int smax = 0;
-    for (int i = 0; i < nt; ++i) {
-        int s = 0;
-        // number of types = sum of block sizes is constant; use nb of the finest term
-        s = T[i].nb;
-        smax = max(smax, s);
-    }
-    if ((int64_t)bitlen64(N + (uint64_t)smax) * smax <= 62) {
+    for (int i = 0; i < nt; ++i) smax = max(smax, (int)T[i].nb);   // the finest partition: s blocks
+    const int bits = bitlen64(N + (uint64_t)smax) * smax;
+    if (bits <= 62) {
         int64_t tot = 0;
         for (int i = 0; i < nt; ++i) {
             int64_t pr = T[i].coef;
             for (int bb = 0; bb < T[i].nb; ++bb) pr *= Z[T[i].mask[bb]];
             tot += pr;
         }
-        return (u128)(uint64_t)tot;       // the count is non-negative
+        out = (u128)(uint64_t)tot;       // the count is non-negative
+        return true;
     }
-    // signed 128-bit (two's complement); flag when the bound fails
-    if ((int64_t)bitlen64(N + (uint64_t)smax) * smax > 126) ovf = true;
-    u128 tot = 0;
+    if (bits > 126) return false;
+    u128 tot = 0;                        // signed 128-bit (two's complement)
     for (int i = 0; i < nt; ++i) {
         const bool neg = T[i].coef < 0;
         u128 pr = (u128)(uint64_t)(neg ? -(int64_t)T[i].coef : T[i].coef);
         for (int bb = 0; bb < T[i].nb; ++bb) pr *= (u128)(uint64_t)Z[T[i].mask[bb]];
         tot = neg ? tot - pr : tot + pr;
     }
-    return tot;
+    out = tot;
+    return true;
 }
 
 template <int NP>
@@ -1660,8 +1661,7 @@ __global__ void __launch_bounds__(kCoreWarps * 32) core_kernel(GraphDev G, Orien
             bool o = false;
             u128 f;
             const int nt = __ldg(TD.cnt + pi);
-            if (nt >= 0) f = fc_partition(vloc, q, TD.terms + __ldg(TD.off + pi), nt, o);
-            else {
+            if (nt < 0 || !fc_partition(vloc, q, TD.terms + __ldg(TD.off + pi), nt, f)) {
                 const FringeProg fp = P.prog[pi];
                 f = fc_dispatch<FSGC_FC_STACK>(vloc, q, fp, o);
             }
@@ -1758,18 +1758,21 @@ __global__ void __launch_bounds__(kCoreWarps * 32) core_kernel(GraphDev G, Orien
     block_publish<NP>(acc, nmatch, S);
 }
 
+// SM count of the current device (cached per device)
 int sm_count() {
-    static int n = 0;
-    if (!n) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
-        if (n <= 0) n = 148;
-    }
+    static std::mutex mu;
+    static std::map<int, int> cache;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    std::lock_guard<std::mutex> lock(mu);
+    auto it = cache.find(dev);
+    if (it != cache.end()) return it->second;
+    int n = 0;
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    if (n <= 0) n = 148;
+    cache[dev] = n;
     return n;
 }
-
-constexpr int kWarps = 4;
 
 // tuning knobs (environment, read once): experiments only, defaults are the
 // tuned values
@@ -1819,23 +1822,35 @@ const void* big_support_kernel(int* warps, size_t* bytes, int cap) {
     return (const void*)support_hash_kernel<FSGC_SUP_CAP>;
 }
 
-// resident blocks per SM of a kernel (cached per function / block / smem)
+// resident blocks per SM of a kernel on the current device (cached per
+// device / function / block / smem); raises the kernel's dynamic shared
+// memory opt-in on that device first (cudaFuncSetAttribute is per device).
+// 0 when the opt-in fails (the launch would fail: the caller reports it).
 int occupancy(const void* fn, int threads, size_t smem) {
     static std::mutex mu;
-    static std::map<std::tuple<const void*, int, size_t>, int> cache;
+    static std::map<std::tuple<int, const void*, int, size_t>, int> cache;
+    static std::map<std::pair<int, const void*>, size_t> optin;
+    int dev = 0;
+    cudaGetDevice(&dev);
     std::lock_guard<std::mutex> lock(mu);
-    auto key = std::make_tuple(fn, threads, smem);
+    auto key = std::make_tuple(dev, fn, threads, smem);
     auto it = cache.find(key);
     if (it != cache.end()) return it->second;
-    int n = 0;
     // the opt-in limit only grows (a plan with less shared memory must not
     // lower it below what an earlier plan of the same kernel launches with)
-    static std::map<const void*, size_t> optin;
-    if (smem > optin[fn]) {   // (static + dynamic above 48 KB needs the opt-in)
-        cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        optin[fn] = smem;
+    size_t& lim = optin[std::make_pair(dev, fn)];
+    if (smem > lim) {   // (static + dynamic above 48 KB needs the opt-in)
+        if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess) {
+            cudaGetLastError();
+            return 0;
+        }
+        lim = smem;
     }
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, threads, smem);
+    int n = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&n, fn, threads, smem) != cudaSuccess) {
+        cudaGetLastError();
+        return 0;
+    }
     n = std::max(n, 1);
     cache[key] = n;
     return n;

@@ -13,6 +13,11 @@
         }                                                                            \
     } while (0)
 
+// the library's own stream-ordered memory pool on the current device
+// (graph.cu): load temporaries are cached there, not in the device's default
+// pool, so the host application's allocators are not affected
+cudaMemPool_t fsgc_device_pool();
+
 template <typename T>
 struct DevBuf {
     T* ptr = nullptr;
@@ -27,7 +32,9 @@ struct DevBuf {
         stream = s;
         count = n;
         if (n == 0) return cudaSuccess;
-        return cudaMallocAsync((void**)&ptr, n * sizeof(T), s);
+        cudaMemPool_t pool = fsgc_device_pool();
+        if (!pool) return cudaErrorInitializationError;
+        return cudaMallocFromPoolAsync((void**)&ptr, n * sizeof(T), pool, s);
     }
     void release() {
         if (ptr) cudaFreeAsync(ptr, stream);

@@ -17,6 +17,7 @@
 #include <atomic>
 #include <mutex>
 #include <set>
+#include <map>
 #include <cstdlib>
 #include <vector>
 #include <algorithm>
@@ -238,24 +239,33 @@ int grid_for(int64_t work) {
     return (int)g;
 }
 
-// The build's temporaries come from the device's default stream-ordered pool.
-// With its default release threshold (0) every synchronisation hands the freed
-// pages back to the driver and the next load maps them again; keep up to
-// 8 GiB cached instead (once per device).
-cudaError_t keep_pool_memory(int dev) {
-    static std::mutex mu;
-    static std::set<int> done;
-    std::lock_guard<std::mutex> lock(mu);
-    if (done.count(dev)) return cudaSuccess;
-    cudaMemPool_t pool;
-    cudaError_t e = cudaDeviceGetDefaultMemPool(&pool, dev);
-    if (e != cudaSuccess) return e;
-    uint64_t keep = 8ull << 30;
-    e = cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
-    if (e == cudaSuccess) done.insert(dev);
-    return e;
-}
 }  // namespace
+
+// The build's temporaries (and the graph arrays) come from a private
+// stream-ordered pool per device.  Its release threshold keeps up to
+// FSGC_POOL_KEEP_BYTES (default 8 GiB) of freed pages mapped, so a load that
+// follows a free (the e2e loop) does not map them again; the device's default
+// pool -- which other libraries in the process may use -- is left untouched.
+cudaMemPool_t fsgc_device_pool() {
+    static std::mutex mu;
+    static std::map<int, cudaMemPool_t> pools;
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) return nullptr;
+    std::lock_guard<std::mutex> lock(mu);
+    auto it = pools.find(dev);
+    if (it != pools.end()) return it->second;
+    cudaMemPoolProps props = {};
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = dev;
+    cudaMemPool_t pool = nullptr;
+    if (cudaMemPoolCreate(&pool, &props) != cudaSuccess) return nullptr;
+    uint64_t keep = 8ull << 30;
+    if (const char* v = getenv("FSGC_POOL_KEEP_BYTES")) keep = strtoull(v, nullptr, 10);
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+    pools[dev] = pool;
+    return pool;
+}
 
 extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, int on_device,
                                void* stream_, fsgc_graph** out) {
@@ -267,7 +277,7 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
     cudaStream_t st = (cudaStream_t)stream_;
     int dev = 0;
     FSGC_CUDA(cudaGetDevice(&dev));
-    FSGC_CUDA(keep_pool_memory(dev));
+    if (!fsgc_device_pool()) FSGC_FAIL(FSGC_ERR_CUDA, "fsgc_load_graph: cannot create the memory pool");
 
     int B = 1;
     while ((1ll << B) < n) ++B;
@@ -323,6 +333,10 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
     if (K > 0) M = hv[0];
     const int bad = (int)hv[1];
     if (bad) FSGC_FAIL(FSGC_ERR_INVALID, "edge list contains a vertex id outside [0, %lld)", (long long)n);
+    // the counting kernels index oriented edges (int32) and CSR positions
+    // (uint32) in 32 bits: 2m must stay below 2^32
+    if (M / 2 >= (1ll << 31))
+        FSGC_FAIL(FSGC_ERR_INVALID, "graph has %lld distinct edges; the limit is 2^31 - 1", (long long)(M / 2));
     kb.release();
 
     // 4 degrees of the original ids

@@ -38,6 +38,30 @@ def count_all(g, pats, **kw):
 _cache = {}
 
 
+# the support pass's two algorithms: the merge kernel (graphs below 2^20
+# edges by default) and the wedge-hash kernels (every larger graph: configs[2],
+# [3], [4]) -- FSGC_SUP_HASH_MIN_M is read at every fsgc_load_graph
+SUP_MODES = {"merge": str(1 << 40), "wedge-hash": "0"}
+
+
+@pytest.fixture(params=sorted(SUP_MODES))
+def sup_mode(request, monkeypatch):
+    monkeypatch.setenv("FSGC_SUP_HASH_MIN_M", SUP_MODES[request.param])
+    return request.param
+
+
+_ofc_cache = {}
+
+
+def oracle_fc(key, gadj, P):
+    """oracle.fringe_count, memoised per (graph key, pattern) across the
+    support-mode parametrisations"""
+    k = (key, P.name, P.core)
+    if k not in _ofc_cache:
+        _ofc_cache[k] = oracle.fringe_count(gadj, P.n, P.edges, P.core)
+    return _ofc_cache[k]
+
+
 def workload(name):
     if name not in _cache:
         n, e = workload_edges(name)
@@ -100,7 +124,7 @@ def test_fig2_paper_values():
 
 
 @pytest.mark.parametrize("seed", range(3))
-def test_all_small_patterns_random_graphs(seed):
+def test_all_small_patterns_random_graphs(seed, sup_mode):
     """All 31 connected patterns <= 5 vertices on random graphs vs mode-1
     brute force (Sec. 3.4's exhaustive check, on the GPU path)."""
     rng = random.Random(seed)
@@ -121,7 +145,7 @@ PL2K_PATTERNS = ["1-tailed-triangle", "2-tailed-triangle", "3-tailed-triangle", 
                  "tricore+6f", "c4core+2f", "clique5", "cycle5"]
 
 
-def test_pl2k_named_patterns():
+def test_pl2k_named_patterns(sup_mode):
     """configs[0] graph (2,000 vertices / 10,000 edges) -- every named pattern
     vs the oracle's core+fringe mode (itself pinned to brute force)."""
     n, e, (_, _, _, gadj) = workload("pl2k")
@@ -129,7 +153,7 @@ def test_pl2k_named_patterns():
     pats = [PATTERNS[x] for x in PL2K_PATTERNS]
     res = count_all(g, [F.compile_named(P) for P in pats])
     for P, r in zip(pats, res):
-        want = oracle.fringe_count(gadj, P.n, P.edges, P.core)
+        want = oracle_fc("pl2k", gadj, P)
         assert not r.overflow and r.count == want, (P.name, r.count, want)
 
 
@@ -162,7 +186,7 @@ def test_batch_equals_single_and_shards_partition():
         assert raws == [r.raw for r in batch]
 
 
-def test_internet_full_size_bench_config():
+def test_internet_full_size_bench_config(sup_mode):
     """configs[1] at full size, in the launch configuration bench.py times
     (one batched pass over the 4 k-tailed triangles): every count exact."""
     n, e, (_, _, _, gadj) = workload("internet")
@@ -170,7 +194,7 @@ def test_internet_full_size_bench_config():
     pats = [PATTERNS[f"{k}-tailed-triangle"] for k in range(1, 5)]
     res = F.fsgc_count(g, [F.compile_named(P) for P in pats])
     for P, r in zip(pats, res):
-        assert r.count == oracle.fringe_count(gadj, P.n, P.edges), P.name
+        assert r.count == oracle_fc("internet", gadj, P), P.name
 
 
 @pytest.mark.parametrize("wl", ["internet", "rmat16"])
@@ -393,7 +417,7 @@ def test_count_distributed_two_ranks_gloo_on_one_gpu():
     assert got == want
 
 
-def test_venn_term_table_tiers_vs_oracle():
+def test_venn_term_table_tiers_vs_oracle(sup_mode):
     """Triangle- and 4-clique-core counts through the Venn term table in all
     three arithmetic tiers -- 64-bit (small leaf triangles), 128-bit and the
     checked Listing 5 fallback (the hub triangle: 13 fringes over ~2^11-sized
@@ -423,10 +447,10 @@ def test_venn_term_table_tiers_vs_oracle():
     res = F.fsgc_count(g, [F.compile_named(P) for P in pats])
     assert res[0].count is not None and res[0].count >= 1 << 100
     for P, r in zip(pats, res):
-        assert not r.overflow and r.count == oracle.fringe_count(gadj, P.n, P.edges, P.core), P.name
+        assert not r.overflow and r.count == oracle_fc("venn-tiers", gadj, P), P.name
 
 
-def test_k_tailed_triangles_rmat16_closed_form():
+def test_k_tailed_triangles_rmat16_closed_form(sup_mode):
     """RMAT-16 (hubs of degree ~6k next to leaf edges): the edge-core pass runs
     its 64- and 128-bit term-table tiers side by side in one block; every
     k-tailed triangle count must equal the closed form sum over triangles of
@@ -440,7 +464,10 @@ def test_k_tailed_triangles_rmat16_closed_form():
     again = F.fsgc_count(g, pats)
     assert [r.raw for r in batch] == [r.raw for r in again]
     for k in ks:
-        want = oracle.k_tailed_triangles(gadj, k)
+        key = ("rmat16-ktt", k)
+        if key not in _ofc_cache:
+            _ofc_cache[key] = oracle.k_tailed_triangles(gadj, k)
+        want = _ofc_cache[key]
         assert not batch[k - 1].overflow and batch[k - 1].count == want, k
         assert F.fsgc_count(g, [pats[k - 1]])[0].count == want, k
 
@@ -491,3 +518,50 @@ def test_rmat26_full_size_wedge_hash_equals_merge():
     b = _one_count_subprocess("rmat26", names, {"FSGC_SUP_MERGE_ONLY": "1"})
     assert a == b, (a, b)
     assert 0 < a["triangle"] < (1_051_923_859 ** 1.5)
+
+
+# ------------------------------------------------ hub-heavy RMAT, symmetry broken
+# The bench configurations count with symmetry breaking on skewed graphs; the
+# full counts of those kernel paths (triangle-core kernel with hubs, general
+# core kernel heavy roots / warp paths / hub bitmaps, both support algorithms)
+# against the C oracle (oracle/cfast.py: every injective core map, explicit
+# Venn, Listing 5; pinned to the Python oracle and closed forms).
+_coracle = {}
+
+
+def _rmat_case(scale):
+    from oracle.cfast import simple_csr
+    key = ("rmat", scale)
+    if key not in _coracle:
+        n = 1 << scale
+        e = rmat_edges_np(scale, 16, seed=9)
+        _coracle[key] = (n, e, simple_csr(n, e))
+    return _coracle[key]
+
+
+def _c_count(scale, P):
+    from oracle.cfast import fringe_count_c
+    key = (scale, P.name)
+    if key not in _coracle:
+        n, e, csr = _rmat_case(scale)
+        _coracle[key] = fringe_count_c(csr, P.n, P.edges, P.core)[0]
+    return _coracle[key]
+
+
+RMAT_CASES = [
+    (12, ["triangle", "1-tailed-triangle", "3-tailed-triangle", "tricore+1f", "tricore+3f", "tricore+6f"]),
+    (8, ["fig4"]),
+    (9, ["clique4", "k4core+2f", "diamondcore+3f", "cycle4", "c4core+2f", "diamond"]),
+]
+
+
+@pytest.mark.parametrize("case", range(len(RMAT_CASES)))
+def test_rmat_hubs_symmetry_broken_vs_c_oracle(case, sup_mode):
+    scale, names = RMAT_CASES[case]
+    n, e, _ = _rmat_case(scale)
+    g = F.fsgc_load_graph(e, n)
+    pats = [PATTERNS[x] for x in names]
+    res = F.fsgc_count(g, [F.compile_named(P) for P in pats])
+    for P, r in zip(pats, res):
+        want = _c_count(scale, P)
+        assert not r.overflow and r.count == want, (scale, P.name, r.count, want)

@@ -366,3 +366,75 @@ def test_partition_lattice_identity_equals_listing5():
                 term *= (-1) ** (len(B) - 1) * factorial(len(B) - 1) * Z[mask]
             tot += term
         assert tot == oracle.fc(list(venn), q, anch, [1] * s)
+
+
+# ------------------------------------------------------------ the C oracle (oracle/cfast.py)
+# The C transcription of mode 2 is pinned to the pinned Python oracle on
+# every small pattern, and to closed forms at sizes the Python oracle does
+# not reach (RMAT graphs with hubs).
+
+def test_c_oracle_equals_python_oracle_all_small_patterns():
+    from oracle.cfast import fringe_count_c, simple_csr
+    for seed in range(3):
+        n = 12 + 2 * seed
+        edges, g = rand_graph(n, 0.4, seed + 40)
+        csr = simple_csr(n, edges)
+        pats = all_connected_patterns(5) + [PATTERNS[x] for x in
+                                            ("fig4", "k4core+6f", "tricore+6f", "c4core+4f", "diamondcore+5f",
+                                             "4-tailed-triangle", "6-star")]
+        for P in pats:
+            assert fringe_count_c(csr, P.n, P.edges, P.core)[0] == oracle.fringe_count(g, P.n, P.edges, P.core), P
+
+
+def test_c_oracle_root_sums_equal_python_oracle():
+    from oracle.cfast import root_raw_sum_c, simple_csr
+    n = 16
+    edges, g = rand_graph(n, 0.35, 7)
+    csr = simple_csr(n, edges)
+    for name in ("tricore+3f", "1-tailed-triangle", "k4core+2f", "c4core+2f"):
+        P = PATTERNS[name]
+        dec = oracle.decompose(P.n, P.edges, P.core)
+        for pv in dec.core:
+            roots = [1, 5, 9]
+            want = sum(oracle.root_raw_sum(g, P.n, P.edges, P.core, pv, r) for r in roots)
+            assert root_raw_sum_c(csr, P.n, P.edges, P.core, pv, roots)[0] == want, (name, pv)
+
+
+def test_c_oracle_closed_forms_on_rmat():
+    """RMAT scale 11 (hubs of degree ~800): k-tailed triangles = sum over
+    triangles of C(deg x - 2, k) (oracle.k_tailed_triangles, itself pinned),
+    k-stars = sum C(deg, k), triangles = trace(A^3) / 6, edges = m."""
+    import scipy.sparse as sp
+    from inputs.graphs import rmat_edges_np
+    from oracle.cfast import fringe_count_c, simple_csr
+    n = 1 << 11
+    e = rmat_edges_np(11, 8, seed=3)
+    csr = simple_csr(n, e)
+    offs, adj = csr
+    g = oracle.csr_to_adjacency(offs, adj)
+    deg = np.diff(offs)
+    A = sp.csr_matrix((np.ones(len(adj), dtype=np.int64), adj, offs), shape=(n, n))
+    tri = int((A @ A).multiply(A).sum()) // 6
+    assert fringe_count_c(csr, 3, PATTERNS["triangle"].edges)[0] == tri
+    assert fringe_count_c(csr, 2, PATTERNS["edge"].edges)[0] == len(adj) // 2
+    for k in (2, 4):
+        P = PATTERNS[f"{k}-star"]
+        assert fringe_count_c(csr, P.n, P.edges)[0] == sum(comb(int(d), k) for d in deg)
+    for k in (1, 3):
+        P = PATTERNS[f"{k}-tailed-triangle"]
+        assert fringe_count_c(csr, P.n, P.edges)[0] == oracle.k_tailed_triangles(g, k)
+        # the same pattern with the triangle forced as the core (Def. 3.1: any
+        # valid core gives the same count)
+        assert fringe_count_c(csr, P.n, P.edges, core=(0, 1, 2))[0] == oracle.k_tailed_triangles(g, k)
+
+
+def test_c_oracle_overflow_is_flagged():
+    """a star with 200,000 leaves: C(200000, 9) > 2^128 must raise, C(n, 7)
+    is exact"""
+    from oracle.cfast import fringe_count_c, simple_csr
+    L = 200000
+    e = np.stack([np.zeros(L, dtype=np.int64), np.arange(1, L + 1)], axis=1)
+    csr = simple_csr(L + 1, e)
+    assert fringe_count_c(csr, 8, star(7).edges)[0] == comb(L, 7)
+    with pytest.raises(OverflowError):
+        fringe_count_c(csr, 10, star(9).edges)
