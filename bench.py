@@ -2,28 +2,35 @@
 """Benchmark of the Fringe-SGC hot path on B200 (driver contract).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl fsgc|reference]
-                    [--workload internet|pl2k|rmat22|pl10m|rmat26]
+                    [--workload rmat26|internet|pl2k|rmat22|rmat16|pl10m|...]
+                    [--no-e2e] [--no-cpu-baseline] [--no-per-config]
 
-One STEP = one pass of the whole hot path (core matching + Venn diagrams +
-fringe counting + 128-bit reduction, and for N>1 the one all-reduce) over
-the workload's graph for all of its patterns.  Default workload: BASELINE.json
-configs[1] -- k-tailed triangles k = 1..4 on the synthetic Internet-like graph
-(124,651 vertices / 193,620 edges); the four patterns share the edge core and
-are counted in ONE batched pass.
+Headline workload (default): BASELINE.json configs[4], the largest
+configuration that fits one GPU -- triangle cores with fringes on RMAT scale
+26 (2^26 vertices, 1.07e9 raw / 1.05e9 distinct edges, 4.9e10 triangles), the
+core forced to the triangle (R13).  All its patterns share the
+triangle core, so one STEP = the per-edge support pass + ONE triangle-core
+listing pass (core matching + Venn diagrams + fringe counting + 128-bit
+reduction; for N>1 the support all-reduce and the one 128-bit all-reduce).
 
 value       core matches / s, device-timed (CUDA events on the launching
             stream), graph resident in HBM, L2 flushed (256 MiB write) before
-            every timed step; N>1: max over ranks.  core matches = core
-            instances in the graph x patterns (edge core: m per pattern).
+            every timed step; N>1: max over ranks.  core matches = the
+            DISTINCT core instances the step enumerates (each triangle once,
+            however many patterns share the pass).  ``edges_per_s`` = m / step
+            time (the paper's Sec. 6 throughput).
 e2e         same metric through the public API from HOST buffers: pinned
-            edge list -> fsgc_load_graph (H2D + CSR build on the GPU) ->
-            fsgc_count -> counts on the host, every step.
-roofline    dominant kernel (the core/Venn/fc kernel): algorithmic bytes per
-            launch / its CUDA-event duration, against
-            the measured HBM copy bandwidth (MEASURED_PEAKS.json).
-cpu_baseline  the oracle (oracle/, unmodified) on a bounded sample of the
-            same workload on the host cores, same unit.
---impl reference  the oracle as the reference arm (CPU), see DESIGN.md.
+            edge list -> fsgc_load_graph (H2D + CSR build) -> fsgc_count ->
+            counts on the host, every step.
+roofline    dominant kernel: algorithmic bytes per launch (DESIGN.md Sec. 5,
+            from the graph's own degree statistics) / its CUDA-event duration,
+            against the measured HBM copy bandwidth (MEASURED_PEAKS.json).
+per_config  configs[0..3] (and the RMAT-26 edge-core decomposition): count
+            time of the batched pass and of every pattern alone, core
+            matches/s and edges/s, per pattern x graph.
+cpu_baseline  the oracle (oracle/cfast.py, C with OpenMP on all host cores,
+            unmodified) on a bounded sample of the same workload, same unit.
+--impl reference  the oracle as the reference arm.
 """
 import argparse
 import json
@@ -43,6 +50,11 @@ METRIC = "count time (s) and core matches/s per pattern×graph at 1/2/4/8 B200"
 UNIT = "core matches/s"
 
 WORKLOAD_DESC = {
+    "rmat26": "triangle cores with fringes (core forced to the triangle: triangle, 1..4 tails on one "
+              "vertex, tails on two vertices, a wedge fringe) on RMAT scale 26, 1.07B raw / 1.05B distinct "
+              "edges (BASELINE configs[4])",
+    "rmat26-edge": "triangle and k-tailed triangles (k=1..4) decomposed to the edge core (Sec. 3.4 "
+                   "heuristic) on RMAT scale 26 (configs[4] graph)",
     "internet": "k-tailed triangles k=1..4 on synthetic Internet-like power-law graph, "
                 "124,651 V / 193,620 E (BASELINE configs[1])",
     "pl2k": "tailed triangle on synthetic power-law graph 2,000 V / 10,000 E (configs[0])",
@@ -50,21 +62,24 @@ WORKLOAD_DESC = {
     "rmat16": "4-clique cores with 1-6 and a diamond core with 1 mixed fringe on RMAT scale 16 "
               "(configs[2] patterns; Table 1's rmat16.sym scale)",
     "pl10m": "Fig. 4 16-vertex/25-edge pattern on synthetic power-law graph, 10M edges (configs[3])",
-    "rmat26": "triangle and k-tailed triangles (k=1..4) on RMAT scale 26, 1.07B raw / 1.05B "
-              "distinct edges (configs[4] graph; patterns decomposed to the edge core)",
 }
+
+# per_config block of the default run: (workload, reps per timing)
+PER_CONFIG = [("pl2k", 20), ("internet", 20), ("rmat16", 2), ("rmat22", 3), ("pl10m", 3), ("rmat26-edge", 2)]
 
 
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=200)
-    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="fsgc", choices=["fsgc", "reference"])
-    ap.add_argument("--workload", default="internet", choices=list(WORKLOAD_DESC))
+    ap.add_argument("--workload", default="rmat26", choices=list(WORKLOAD_DESC))
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--cpu-budget", type=float, default=12.0, help="seconds of oracle work")
+    ap.add_argument("--no-per-config", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work")
     return ap.parse_args()
 
 
@@ -145,88 +160,252 @@ def ncu_traffic(workload, kernel):
     return None
 
 
+def graph_key(name):
+    return "rmat26" if name.startswith("rmat26") else name
+
+
 def load_workload(name, device):
+    """(n, edges, patterns): RMAT graphs generated with torch on ``device``
+    (int32 tensor), the others with numpy (int64 array)."""
     from inputs import workload_edges
     from inputs.patterns import CONFIG_PATTERNS, PATTERNS
-    if name in ("rmat16", "rmat22", "rmat26"):
-        n, e = workload_edges(name, device=device)
+    gk = graph_key(name)
+    if gk.startswith("rmat"):
+        n, e = workload_edges(gk, device=device if device is not None else "cpu")
     else:
-        n, e = workload_edges(name)
-    pats = [PATTERNS[x] for x in CONFIG_PATTERNS[name]]
-    return n, e, pats
+        n, e = workload_edges(gk)
+    return n, e, [PATTERNS[x] for x in CONFIG_PATTERNS[name]]
+
+
+def simple_csr_torch(n, e):
+    """The simple graph of an edge list as a CSR with sorted adjacency lists
+    and ORIGINAL ids (loops dropped, duplicates merged) -- plain torch
+    sort/unique on the edge tensor's device, then to host numpy.  Input
+    preparation of the oracle's CPU baseline for graphs too large for numpy
+    (the oracle's own oracle.cfast.simple_csr builds the same arrays)."""
+    import torch
+    a = e[:, 0].to(torch.int64)
+    b = e[:, 1].to(torch.int64)
+    ok = a != b
+    a, b = a[ok], b[ok]
+    key = torch.unique(torch.cat([a * n + b, b * n + a]))
+    src = key // n
+    offs = torch.zeros(n + 1, dtype=torch.int64, device=key.device)
+    offs[1:] = torch.cumsum(torch.bincount(src, minlength=n), 0)
+    return offs.cpu().numpy(), (key % n).to(torch.int32).cpu().numpy()
+
+
+def host_csr(n, e):
+    import numpy as np
+    if isinstance(e, np.ndarray):
+        from oracle.cfast import simple_csr
+        return simple_csr(n, e)
+    return simple_csr_torch(n, e)
+
+
+def oracle_cpu_sample(csr, pats, budget_s, seed=0, max_deg=20000, nroots=None):
+    """The unmodified C oracle (oracle.cfast.root_raw_sum_c: every core map
+    with the root pattern vertex on the sampled graph vertices, explicit Venn,
+    Listing 5; OpenMP on all host cores) on seeded random root vertices of
+    degree <= max_deg, in batches until ``budget_s`` seconds are spent (or on
+    exactly ``nroots`` roots).  Returns (core matches processed, seconds,
+    roots, threads): core matches = core maps / |Aut(core)|, the unit of the
+    GPU line."""
+    import numpy as np
+    import oracle
+    from oracle.cfast import root_raw_sum_c
+    offs, _ = csr
+    n = len(offs) - 1
+    deg = np.diff(offs)
+    rng = np.random.default_rng(seed)
+    cand = np.nonzero((deg >= 1) & (deg <= max_deg))[0]
+    roots = rng.permutation(cand)[: (nroots if nroots is not None else 2_000_000)]
+    threads = os.cpu_count() or 1
+    decs = []
+    for P in pats:
+        dec = oracle.decompose(P.n, P.edges, P.core)
+        cs = list(dec.core)
+        rel = {v: i for i, v in enumerate(cs)}
+        cedges = [(rel[x], rel[y]) for x, y in P.edges if x in rel and y in rel]
+        decs.append((P, cs[0], oracle.automorphism_count(len(cs), cedges)))
+    matches, done, t0 = 0.0, 0, time.perf_counter()
+    batch = 256
+    while done < len(roots):
+        chunk = roots[done:done + batch]
+        for P, pv, autc in decs:
+            _, maps = root_raw_sum_c(csr, P.n, P.edges, P.core, pv, chunk, threads=threads)
+            matches += maps / autc
+        done += len(chunk)
+        if nroots is None and time.perf_counter() - t0 >= budget_s:
+            break
+        batch = min(batch * 2, 1 << 16)
+    return matches, time.perf_counter() - t0, done, threads
 
 
 # ------------------------------------------------------------------ oracle arm
 
-def oracle_prepare(n, edges, pats):
-    """The oracle's own graph (degree-ordered CSR by definition) and pattern
-    decompositions, built once outside the timed sample."""
-    import oracle
-    offs, adj, _ = oracle.degree_ordered_csr(n, edges)
-    gadj = oracle.csr_to_adjacency(offs, adj)
-    decs = [(P, list(oracle.decompose(P.n, P.edges, P.core).core)) for P in pats]
-    return gadj, decs
-
-
-def oracle_sample(prep, budget_s, seed=0, sample=None):
-    """Run the unmodified oracle (core+fringe mode, per root vertex, no
-    symmetry breaking) on root vertices in a seeded random order until
-    ``budget_s`` seconds are spent (or on exactly ``sample`` vertices).
-    Returns (core instances processed, seconds, vertices)."""
-    import oracle
-    gadj, decs = prep
-    verts = list(range(len(gadj)))
-    random.Random(seed).shuffle(verts)
-    if sample is not None:
-        verts = verts[:sample]
-    maps = 0.0
-    done = 0
-    t0 = time.perf_counter()
-    for r in verts:
-        for P, cs in decs:
-            oracle.root_raw_sum(gadj, P.n, P.edges, P.core, cs[0], r)
-            if len(cs) == 2:       # edge core: deg(r) core maps rooted at r, 2 per instance
-                maps += len(gadj[r]) / 2.0
-            elif len(cs) == 1:
-                maps += 1
-        done += 1
-        if sample is None and time.perf_counter() - t0 >= budget_s:
-            break
-    return maps, time.perf_counter() - t0, done
-
-
 def run_reference(args, rank, world):
+    """--impl reference: the oracle (C, all host cores) timed on the host on
+    the same workload, metric and unit; rank 0 only."""
     if rank != 0:
         return
-    n, e, pats = load_workload(args.workload, None)
-    if hasattr(e, "cpu"):
-        e = e.cpu().numpy()
+    dev = None
+    try:
+        import torch
+        if torch.cuda.is_available():
+            dev = torch.device("cuda", 0)
+    except ImportError:
+        pass
+    n, e, pats = load_workload(args.workload, dev)
+    csr = host_csr(n, e)
+    del e
     # size one step so the whole run stays within a few minutes
-    prep = oracle_prepare(n, e, pats)
-    step_budget = max(0.2, 120.0 / max(1, args.steps + args.warmup))
-    _, _, nv = oracle_sample(prep, step_budget, seed=99)
-    nv = max(1, nv)
-    vals, secs = [], []
+    step_budget = max(0.5, 150.0 / max(1, args.steps + args.warmup))
+    _, _, nr, _ = oracle_cpu_sample(csr, pats, step_budget, seed=99)
+    vals, secs, threads = [], [], 1
     for s in range(args.warmup + args.steps):
-        maps, dt, _ = oracle_sample(prep, 0, seed=s, sample=nv)
+        maps, dt, _, threads = oracle_cpu_sample(csr, pats, 0, seed=s, nroots=nr)
         if s >= args.warmup:
             vals.append(maps)
             secs.append(dt)
     value = sum(vals) / sum(secs)
+    sample = (f"{nr} seeded random root vertices (degree <= 20000) per step x {len(pats)} patterns, "
+              f"C oracle root sums, {threads} OpenMP threads")
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * sum(secs) / len(secs),
-        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "python-int",
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u128/u256 (C oracle)",
         "data": "synthetic",
         "config": {"workload": WORKLOAD_DESC[args.workload], "patterns": [p.name for p in pats]},
-        "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
-                         "sample": f"{nv} seeded random root vertices per step x {len(pats)} patterns"},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
 
 
+# ------------------------------------------------------------------ roofline
+
+def listing_stats(n, e):
+    """Degree-orientation statistics of the graph (plain torch on the edge
+    tensor's device): m, sum over oriented edges (a, b) of the tail length of
+    N+(a) after b (the listing kernels' streamed elements), and the merge
+    kernel's sum of out(a) + out(b)."""
+    import torch
+    dev = e.device if hasattr(e, "device") else "cpu"
+    et = e if hasattr(e, "device") else torch.from_numpy(e)
+    a = et[:, 0].to(torch.int64)
+    b = et[:, 1].to(torch.int64)
+    ok = a != b
+    lo = torch.minimum(a[ok], b[ok])
+    hi = torch.maximum(a[ok], b[ok])
+    k = torch.unique(lo * n + hi)
+    del a, b, ok, lo, hi
+    a, b = k // n, k % n
+    del k
+    deg = torch.bincount(a, minlength=n) + torch.bincount(b, minlength=n)
+    rank = torch.empty(n, dtype=torch.int64, device=dev)
+    rank[torch.argsort(deg * n + torch.arange(n, device=dev))] = torch.arange(n, device=dev)
+    ra, rb = rank[a], rank[b]
+    del a, b
+    u, v = torch.minimum(ra, rb), torch.maximum(ra, rb)
+    del ra, rb
+    out = torch.bincount(u, minlength=n)
+    s = torch.argsort(u * n + v)
+    u, v = u[s], v[s]
+    del s
+    oofs = torch.zeros(n + 1, dtype=torch.int64, device=dev)
+    oofs[1:] = torch.cumsum(out, 0)
+    tail = out[u] - (torch.arange(u.numel(), device=dev) - oofs[u]) - 1
+    st = {"m": int(u.numel()), "tail": float(tail.sum()), "merge": float((out[u] + out[v]).sum())}
+    del u, v, tail, oofs, out, deg, rank
+    if dev != "cpu":
+        torch.cuda.empty_cache()
+    return st
+
+
+def support_bytes(st, tri, hash_mode):
+    """listing support pass 44 B per oriented edge (in-entry
+    a, rev, split/oofs/offs of a; table staging and c(b, x) flush) + 4 B per
+    streamed tail element + 8 B per triangle (c(a, c) reduction); merge
+    kernel 40 B per edge + 4 B per merged out-list element"""
+    if hash_mode:
+        return 44.0 * st["m"] + 4.0 * st["tail"] + 8.0 * tri
+    return 40.0 * st["m"] + 4.0 * st["merge"]
+
+
+def tricore_bytes(st, tri):
+    """triangle-core listing pass: 32 B per in-entry (a, rev, split/oofs/offs)
+    + 20 B per in-entry (deg a, c(ab)) + 24 B per N+(b) entry staged (adj, c,
+    deg) + 4 B per tail element + 4 B per triangle (c(a, c))"""
+    return 76.0 * st["m"] + 4.0 * st["tail"] + 4.0 * tri
+
+
 # ------------------------------------------------------------------ GPU arm
+
+def pass_core_matches(F, g, cps):
+    """distinct core instances per step: per pass, the core-match count of its
+    first pattern with the degree filter off (untimed)"""
+    probe = F.fsgc_count(g, cps, no_degree_filter=True)
+    seen = {}
+    for r in probe:
+        seen.setdefault(r.pass_index, r.core_matches)
+    return sum(seen.values()), probe
+
+
+def time_counts(F, g, cps, reps, flush):
+    """device time (ms) of `reps` synchronous fsgc_count calls (min), counts"""
+    import torch
+    best, res = None, None
+    st = torch.cuda.current_stream()
+    for _ in range(reps):
+        flush.fill_(1)
+        torch.cuda.synchronize()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(st)
+        res = F.fsgc_count(g, cps)
+        b.record(st)
+        torch.cuda.synchronize()
+        ms = a.elapsed_time(b)
+        best = ms if best is None else min(best, ms)
+    return best, res
+
+
+def per_config_block(F, dev, flush, skip):
+    """configs[0..3] and the RMAT-26 edge-core decomposition: batched pass
+    time and every pattern alone, per pattern x graph"""
+    import torch
+    out = []
+    for wl, reps in PER_CONFIG:
+        if wl == skip:
+            continue
+        try:
+            n, e, pats = load_workload(wl, dev)
+            g = F.fsgc_load_graph(e, n)
+            del e
+            cps = [F.compile_named(P) for P in pats]
+            cm, _ = pass_core_matches(F, g, cps)
+            time_counts(F, g, cps, 1, flush)                       # warm-up (plans, tables)
+            ms, res = time_counts(F, g, cps, reps, flush)
+            per = {}
+            for P, p, r in zip(pats, cps, res):
+                time_counts(F, g, [p], 1, flush)
+                pms, pr = time_counts(F, g, [p], reps, flush)
+                per[P.name] = {"count": str(r.count) if r.count is not None else None,
+                               "overflow": r.overflow, "count_time_s": pms / 1e3,
+                               "core_matches": pr[0].core_matches,
+                               "core_matches_per_s": pr[0].core_matches / (pms / 1e3)}
+            out.append({"workload": WORKLOAD_DESC[wl], "graph": {"n": n, "m": g.m, "max_degree": g.max_degree},
+                        "batched": {"count_time_s": ms / 1e3, "core_matches": cm,
+                                    "core_matches_per_s": cm / (ms / 1e3), "edges_per_s": g.m / (ms / 1e3),
+                                    "passes": len({r.pass_index for r in res})},
+                        "patterns": per})
+            g.free()
+            del g
+            torch.cuda.empty_cache()
+        except Exception as ex:  # a failing side config must not hide the headline line
+            out.append({"workload": wl, "error": repr(ex)[:300]})
+    return out
+
 
 def main():
     args = parse()
@@ -260,12 +439,11 @@ def main():
     else:
         e_dev = e.contiguous()
         e_host = e_dev.cpu().pin_memory()
+    del e
+    st_graph = listing_stats(n, e_dev)
     g = F.fsgc_load_graph(e_dev, n)
     cps = [F.compile_named(P) for P in pats]
-
-    # core instances per step (graph property, untimed): degree filter off
-    probe = F.fsgc_count(g, cps, no_degree_filter=True, shard_index=0, shard_count=1)
-    core_matches = sum(r.core_matches for r in probe)
+    core_matches, _ = pass_core_matches(F, g, cps)
 
     stream = torch.cuda.current_stream()
     if world > 1:
@@ -297,7 +475,7 @@ def main():
     for _ in range(args.warmup):
         res = step()
     counts = [r.count for r in res]
-    ref = F.fsgc_count(g, cps)                       # the synchronous API agrees
+    ref = F.fsgc_count_distributed(g, cps) if world > 1 else F.fsgc_count(g, cps)   # the synchronous API agrees
     assert [r.count for r in ref] == counts, (counts, [r.count for r in ref])
     torch.cuda.synchronize()
     if world > 1:
@@ -350,58 +528,42 @@ def main():
     value = core_matches / (ms_per_step / 1e3)
     kind_of = {r.pass_index: r.pass_kind for r in res}
 
-    # ---- roofline of the dominant kernel (DESIGN.md "Roofline"): algorithmic
+    # ---- roofline of the dominant kernel (DESIGN.md Sec. 5): algorithmic
     # bytes per launch / CUDA-event duration, against the measured HBM peak
-    offs, adj_h, _ = g.download()
-    deg = np.diff(offs).astype(np.int64)
-    rows = np.repeat(np.arange(n, dtype=np.int64), deg)
-    up = adj_h.astype(np.int64) > rows
-    out = np.bincount(rows[up], minlength=n).astype(np.float64)
-    indeg = deg - out
     m = g.m
     share = 1.0 / world
-    # support pass: wedge-hash part -- per in-entry
-    # (a, b) of a table middle b: 4 B a + 4 B rev + 24 B split/oofs/offs of a,
-    # 4 B per tail element c > b of N+(a) streamed, 4 B per N+(b) entry staged
-    # (+ its c(b, x) flush), 8 B per triangle (the c(a, c) reduction); merge
-    # part -- per heavy-middle edge 40 B + 4 B per merged out-list entry
-    CAP = 4096
-    a_o = rows[up]
-    b_o = adj_h[up].astype(np.int64)
-    oofs_h = np.concatenate([[0], np.cumsum(out)]).astype(np.int64)
-    tail = out[a_o] - (np.arange(len(a_o), dtype=np.int64) - oofs_h[a_o]) - 1
-    ob = out[b_o]
-    light = (ob >= 1) & (ob <= CAP)
-    heavy = ob > CAP
     tri = 0
     if plan is not None and plan.support() is not None:
         tri = int(plan.support().to(torch.int64).sum().item()) // 3
-    mid = (out >= 1) & (out <= CAP) & (indeg >= 1)
-    sup_bytes = (32.0 * float(light.sum()) + 4.0 * float(tail[light].sum()) + 8.0 * float(out[mid].sum())
-                 + 8.0 * tri + 40.0 * float(heavy.sum()) + 4.0 * float((out[a_o] + ob)[heavy].sum()))
-    # fc pass: per root edge 8 B (u,v) + 32 B (4 offsets) + 4 B support
-    fc_bytes = 44.0 * m * share
-    # general / triangle core passes: compulsory graph bytes (CSR + oriented
-    # view + supports read once) -- these kernels are latency/ALU bound
-    graph_bytes = (8.0 * 2 * m + 8.0 * (n + 1) + 8.0 * m + 4.0 * m + 16.0 * n) * share
+    hash_mode = g.m >= int(os.environ.get("FSGC_SUP_HASH_MIN_M", str(1 << 20)))
+    sup_b = support_bytes(st_graph, tri, hash_mode) * share
     names = {0: "vertex_core_kernel", 1: "edge_fc_kernel (Venn + Sec. 3.1 fc, lane per root edge)",
              2: "core_kernel (general core: DFS + min-list Venn + fc)",
-             3: "tri_core_kernel (triangle core: listing + Venn + fc)"}
+             3: "list_*_kernel<tri> (triangle cores: listing by middle vertex + Venn + fc)"}
     kernels = []
     for k in pass_ids:
         kind = kind_of[k]
-        byts = fc_bytes if kind == 1 else (8.0 * (n + 1) * share if kind == 0 else graph_bytes)
+        if kind == 1:
+            byts = 44.0 * m * share
+        elif kind == 3:
+            byts = tricore_bytes(st_graph, tri) * share
+        elif kind == 0:
+            byts = 8.0 * (n + 1) * share
+        else:   # compulsory graph bytes: CSR + oriented view + supports, read once
+            byts = (8.0 * 2 * m + 8.0 * (n + 1) + 8.0 * m + 4.0 * m + 16.0 * n) * share
         kernels.append((names[kind] + f" [pass {k}]", byts, kms_sum[k] / args.steps))
-        if kind != 0:
-            kernels.append((f"support_kernel (per-edge |N(u)&N(v)| by oriented listing) [pass {k}]",
-                            sup_bytes, ams_sum[k] / args.steps))
+        if kind != 0 and ams_sum[k] > 0:
+            kernels.append((("list_*_kernel<support> (per-edge |N(u)&N(v)|, listing by middle vertex)"
+                             if hash_mode else "support_kernel (per-edge |N(u)&N(v)|, merge)") + f" [pass {k}]",
+                            sup_b, ams_sum[k] / args.steps))
     kernels.sort(key=lambda kk: -kk[2])
     peak, peak_src = measured_peaks()
+
     def roof(name, byts, ms):
-        traffic = ncu_traffic(args.workload, name)
+        traffic = ncu_traffic(graph_key(args.workload), name)
         ach = byts / (ms / 1e3) / 1e9 if ms > 0 else 0.0
         return {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
-                "traffic": traffic, "kernel": name, "kernel_ms": ms,
+                "traffic": traffic, "kernel": name, "kernel_ms": ms, "share_of_step": ms / ms_per_step,
                 "algorithmic_bytes_per_launch": byts, "peak_source": peak_src}
 
     # ---- e2e through the public API from pinned host buffers
@@ -409,8 +571,12 @@ def main():
     if not args.no_e2e:
         h2d = e_host.numel() * e_host.element_size()
         d2h = 36 + 16 * 32 + 8
+        del plan, replay
+        if world == 1:
+            del cg
+        torch.cuda.empty_cache()
         tms = []
-        for s in range(3 + min(args.steps, 50)):
+        for s in range(1 + max(1, args.e2e_steps)):
             flush.fill_(s)
             torch.cuda.synchronize()
             if world > 1:
@@ -423,7 +589,7 @@ def main():
             torch.cuda.synchronize()
             assert [x.count for x in r2] == counts
             g2.free()
-            if s >= 3:
+            if s >= 1:
                 tms.append(a.elapsed_time(b))
         et = sum(tms)
         if world > 1:
@@ -432,15 +598,24 @@ def main():
             et = t.item()
         e2e = {"value": core_matches / (et / len(tms) / 1e3), "unit": UNIT,
                "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
-               "ms_per_step": et / len(tms)}
+               "ms_per_step": et / len(tms), "steps": len(tms)}
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        e_np = e if isinstance(e, np.ndarray) else e.cpu().numpy()
-        maps, secs, nv = oracle_sample(oracle_prepare(n, e_np, pats), args.cpu_budget)
-        cpu = {"value": maps / secs, "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": f"{nv} seeded random root vertices x {len(pats)} patterns "
-                         f"({secs:.1f} s, per-root core+fringe oracle, 1 Python thread)"}
+        csr = host_csr(n, e_dev)
+        maps, secs, nr, threads = oracle_cpu_sample(csr, pats, args.cpu_budget)
+        del csr
+        cpu = {"value": maps / secs, "unit": UNIT, "cores": threads, "kind": "oracle",
+               "sample": f"{nr} seeded random root vertices (degree <= 20000) x {len(pats)} patterns "
+                         f"({secs:.1f} s, C oracle root sums: every core map, explicit Venn, Listing 5; "
+                         f"{threads} OpenMP threads)"}
+    del e_dev
+
+    per_config = None
+    if rank == 0 and world == 1 and not args.no_per_config:
+        g.free()
+        torch.cuda.empty_cache()
+        per_config = per_config_block(F, dev, flush, args.workload)
 
     if rank == 0:
         line = {
@@ -448,19 +623,24 @@ def main():
             "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
             "scaling": "strong", "vs_baseline": None, "dtype": "u128", "data": "synthetic",
             "config": {"workload": WORKLOAD_DESC[args.workload], "patterns": [p.name for p in pats],
-                       "graph": {"n": n, "m": m, "max_degree": g.max_degree},
+                       "graph": {"n": n, "m": m, "max_degree": g.max_degree,
+                                 "triangles": tri or None},
                        "core_matches_per_step": core_matches,
                        "count_time_s": ms_per_step / 1e3,
+                       "edges_per_s": m / (ms_per_step / 1e3),
                        "counts": {p.name: str(c) for p, c in zip(pats, counts)},
-                       "l2": "flushed before every timed step (256 MiB write)",
-                       "parallelism": f"{world} GPU(s): graph replicated, root-edge chunks dealt "
-                                      f"round-robin, 1 all-reduce of 128-bit partials"},
+                       "l2": "flushed before every timed step (256 MiB write); graph >> L2",
+                       "parallelism": f"{world} GPU(s): graph replicated, support units and triangle-listing "
+                                      f"units dealt round-robin, support all-reduce + 1 all-reduce of "
+                                      f"128-bit partials"},
+            "edges_per_s": m / (ms_per_step / 1e3),
             "gpu_launches": launches,
             "roofline": roof(*kernels[0]),
             "roofline_other_kernels": [roof(*k) for k in kernels[1:]],
             "clocks": clocks,
             "e2e": e2e,
             "cpu_baseline": cpu,
+            "per_config": per_config,
         }
         print(json.dumps(line), flush=True)
     if world > 1:

@@ -103,6 +103,13 @@ def triangle_core(nf):
     return core_with_fringes("tricore", [(0, 1), (1, 2), (0, 2)], 3, nf, seq)
 
 
+def ktt_tricore(k):
+    """the k-tailed triangle with its triangle FORCED as the core (DESIGN.md
+    R7, R13): k tails on vertex 0, one fringe type, anchor set {0}."""
+    e = [(0, 1), (0, 2), (1, 2)] + [(0, 3 + i) for i in range(k)]
+    return _p(f"{k}-tailed-triangle/tricore", 3 + k, e, core=(0, 1, 2))
+
+
 def c4_core(nf):
     """4-cycle core 0-1-2-3 (forced) + fringes (configs[4])."""
     seq = [(0,), (1,), (2,), (3,), (0, 2), (1, 3)]
@@ -128,6 +135,10 @@ def _build():
     put(fig4())
     for nf in range(1, 7):
         put(k4_core(nf)); put(diamond_core(nf)); put(triangle_core(nf)); put(c4_core(nf))
+    for k in range(2, 5):
+        put(ktt_tricore(k))
+    put(_p("triangle/tricore", 3, [(0, 1), (0, 2), (1, 2)], core=(0, 1, 2)))
+    put(_p("diamond/tricore", 4, DIAMOND_EDGES, core=(0, 1, 2)))
     return P
 
 
@@ -145,10 +156,14 @@ CONFIG_PATTERNS = {
     "rmat22": ["triangle", "diamond"] + [f"{k}-tailed-triangle" for k in range(1, 5)],
     "rmat16": [f"k4core+{f}f" for f in range(1, 7)] + ["diamondcore+1f"],
     "pl10m": ["fig4"],
-    # configs[4]: triangle-with-fringes patterns on RMAT-26 as the compiler
-    # decomposes them (edge core, R13); the forced triangle / 4-cycle
-    # core sets below do not finish a step at this scale (Next)
-    "rmat26": ["triangle"] + [f"{k}-tailed-triangle" for k in range(1, 5)],
+    # configs[4]: triangle cores with fringes on RMAT-26, the core FORCED to
+    # the triangle (R13): every fringe set whose Venn diagram needs
+    # no triple intersection (tails, wedges on two core vertices) -- one
+    # listing pass over the 4.9e10 triangles for all of them
+    "rmat26": ["triangle/tricore", "tricore+1f", "tricore+2f", "2-tailed-triangle/tricore",
+               "3-tailed-triangle/tricore", "4-tailed-triangle/tricore", "diamond/tricore"],
+    # the same patterns decomposed by the Sec. 3.4 heuristic (edge core)
+    "rmat26-edge": ["triangle"] + [f"{k}-tailed-triangle" for k in range(1, 5)],
     "rmat26-forced-cores": [f"tricore+{f}f" for f in range(1, 7)] + [f"c4core+{f}f" for f in range(1, 7)],
 }
 

@@ -21,7 +21,7 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-O3", "-I", CSRC]
 
 SOURCES = ["pattern.cpp", "graph.cu", "count.cu"]
-HEADERS = ["internal.h", "devbuf.cuh", "u128.cuh"]
+HEADERS = ["internal.h", "devbuf.cuh", "u128.cuh", "fc.cuh", "listing.cuh"]
 
 
 def _newer(src, dst):

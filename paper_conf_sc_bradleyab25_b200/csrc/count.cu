@@ -268,7 +268,7 @@ __device__ __noinline__ void block_publish(const AccN<NP> A, unsigned long long 
 // 1-vertex cores (k-stars, the 1- and 2-vertex patterns): one thread per
 // root vertex, Venn = {deg(v)} (Sec. 3 k-star formula generalised by fc).
 template <int NP>
-__global__ void __launch_bounds__(256) vertex_core_kernel(GraphDev G, const CoreProg P, WorkDesc W,
+__global__ void __launch_bounds__(256) vertex_core_kernel(GraphDev G, const __grid_constant__ CoreProg P, WorkDesc W,
                                                           const Sink S) {
     AccN<NP> acc;
     acc.init();
@@ -463,248 +463,6 @@ __global__ void __launch_bounds__(256) support_kernel(GraphDev G, OrientDev O, i
     }
 }
 
-// Wedge-hash part of the support pass: every triangle a < b < c is found
-// from its MIDDLE vertex b.  A warp takes a unit (b, k) from a global atomic
-// queue, stages N+(b) (out(b) <= FSGC_SUP_CAP) in a shared-memory hash table
-// (key -> position in N+(b)), takes the k-th slice of b's in-list
-// N-(b) = {a < b}, and streams, for every a of the slice, the tail of N+(a)
-// after b (the c > b; b's position in N+(a) comes from graph.rev), probing
-// each c in the table.  The tails of the slice are concatenated (warp prefix
-// sum of their lengths) so the 32 lanes always read 32 consecutive virtual
-// elements: coalesced adjacency reads whatever the tail lengths.  A hit is
-// the triangle (a, b, c): c(bc) += 1 in shared memory (flushed per unit),
-// c(ab) += 1 in shared memory (flushed per slice), c(ac) += 1 by a global
-// reduction.  Work: sum_a out(a)^2 / 2 adjacency elements instead of the
-// merge's sum_(a,b) (out(a) + out(b)).
-// Two variants: a small table (out(b) <= CAPW, the many small middles; the
-// slice's tails are concatenated, sup_slice) and a large one (CAPW < out(b)
-// <= CAP: long tails, streamed one at a time, sup_slice_stream).  One warp
-// per unit, its own table sized to out(b) (load factor <= 1/2), no block
-// barriers.
-// FSGC_SUP_BIG (experiments) picks the large-table variant: 0 streamed
-// tails, 4 warps; 1 concatenated tails (sup_slice), 4 warps; 2 streamed, 2 warps
-template <int CAPT, bool STR = (CAPT > FSGC_SUP_CAPW), int NW = (STR ? 4 : 8)>
-struct SupLayout {
-    static constexpr bool STREAM = STR;
-    static constexpr int WARPS = NW;
-    static constexpr int HS = 2 * CAPT;
-    static constexpr size_t table_bytes = (size_t)HS * 4 + (size_t)HS * 2 + (size_t)CAPT * 4;
-    static constexpr size_t slice_bytes = STREAM ? 0 : (size_t)(FSGC_SUP_SEG + 4) * 4 + (size_t)4 * FSGC_SUP_SEG * 4;
-    static constexpr size_t warp_bytes = table_bytes + slice_bytes;
-    static constexpr size_t bytes = WARPS * warp_bytes;
-};
-
-// one warp, one slice [ib0, ib0 + len) of N-(b): tails of N+(a) after b,
-// concatenated; two virtual elements per lane in flight
-__device__ __forceinline__ void sup_slice(const GraphDev& G, const OrientDev& O, const int32_t* __restrict__ rev,
-                                          int* __restrict__ sup, int64_t ib0, int len, int64_t rbase,
-                                          const int32_t* key, const int16_t* kpos, int32_t* cb, int hbits,
-                                          int32_t* pre, uint32_t* q0, uint32_t* da, int32_t* ea, int32_t* cab,
-                                          int lane) {
-    const uint32_t hm = (1u << hbits) - 1;
-    int carry = 0;
-    for (int j0 = 0; j0 < len; j0 += 32) {
-        const int j = j0 + lane;
-        int L = 0;
-        if (j < len) {
-            const int a = __ldg(G.adj + ib0 + j);
-            const int e = __ldg(rev + rbase + j);
-            const int64_t sa = __ldg(O.split + a), oa = __ldg(O.oofs + a);
-            const int64_t q = sa + (e - oa) + 1;
-            L = (int)(__ldg(G.offs + a + 1) - q);
-            q0[j] = (uint32_t)q;
-            da[j] = (uint32_t)(sa - oa);
-            ea[j] = e;
-            cab[j] = 0;
-        }
-        int x = L;                        // inclusive warp scan
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const int y = __shfl_up_sync(FULLMASK, x, o);
-            if (lane >= o) x += y;
-        }
-        if (j < len) pre[j] = carry + x - L;
-        carry += __shfl_sync(FULLMASK, x, 31);
-    }
-    if (lane == 0) pre[len] = carry;
-    __syncwarp();
-    const int total = carry;
-    int lo = 0;                           // monotone: last j with pre[j] <= idx
-    for (int v0 = 0; v0 < total; v0 += 64) {
-        int jj[2], cc[2];
-        uint32_t pp[2];
-        bool ok[2];
-#pragma unroll
-        for (int r = 0; r < 2; ++r) {
-            const int idx = v0 + 32 * r + lane;
-            ok[r] = idx < total;
-            jj[r] = 0; pp[r] = 0; cc[r] = -1;
-            if (ok[r]) {
-                int l2 = lo, hi = len;
-                while (hi - l2 > 1) {
-                    const int mid = (l2 + hi) >> 1;
-                    if (pre[mid] <= idx) l2 = mid; else hi = mid;
-                }
-                lo = l2;
-                jj[r] = l2;
-                pp[r] = q0[l2] + (uint32_t)(idx - pre[l2]);
-                cc[r] = __ldg(G.adj + pp[r]);
-            }
-        }
-#pragma unroll
-        for (int r = 0; r < 2; ++r) {
-            bool hit = false;
-            int kk = -1;
-            if (ok[r]) {
-                uint32_t h = ((uint32_t)cc[r] * 0x9E3779B1u) >> (32 - hbits);
-                int y;
-                while ((y = key[h]) != cc[r] && y != -1) h = (h + 1) & hm;
-                hit = y == cc[r];
-                if (hit) kk = kpos[h];
-            }
-            const unsigned hmask = __ballot_sync(FULLMASK, hit);
-            if (hit) {
-                atomicAdd(&cb[kk], 1);
-                atomicAdd(sup + (pp[r] - da[jj[r]]), 1);
-                const unsigned peers = __match_any_sync(hmask, jj[r]);   // c(a, b): one add per a
-                if ((peers & ((1u << lane) - 1)) == 0) atomicAdd(&cab[jj[r]], __popc(peers));
-            }
-        }
-    }
-    __syncwarp();
-    for (int j = lane; j < len; j += 32)
-        if (cab[j]) atomicAdd(sup + ea[j], cab[j]);
-    __syncwarp();
-}
-
-constexpr int kSupILP = 4;   // tail loads in flight per lane
-
-// one warp, one slice of N-(b) whose tails are long (block tables: the
-// middles of large out-degree): the warp streams one tail at a time, 32
-// consecutive elements per step (two steps in flight), c(a, b) = the hits
-// counted by ballot, one global add per (a, b)
-__device__ __forceinline__ void sup_slice_stream(const GraphDev& G, const OrientDev& O,
-                                                 const int32_t* __restrict__ rev, int* __restrict__ sup,
-                                                 int64_t ib0, int len, int64_t rbase, const int32_t* key,
-                                                 const int16_t* kpos, int32_t* cb, int hbits, int lane) {
-    const uint32_t hm = (1u << hbits) - 1;
-    for (int j0 = 0; j0 < len; j0 += 32) {
-        const int j = j0 + lane;
-        int64_t q = 0, dA = 0;
-        int L = 0, e = 0;
-        if (j < len) {
-            const int a = __ldg(G.adj + ib0 + j);
-            e = __ldg(rev + rbase + j);
-            const int64_t sa = __ldg(O.split + a), oa = __ldg(O.oofs + a);
-            q = sa + (e - oa) + 1;
-            L = (int)(__ldg(G.offs + a + 1) - q);
-            dA = sa - oa;
-        }
-        const int nj = min(32, len - j0);
-        for (int t = 0; t < nj; ++t) {
-            const int64_t qt = __shfl_sync(FULLMASK, q, t);
-            const int Lt = __shfl_sync(FULLMASK, L, t);
-            const int64_t dt = __shfl_sync(FULLMASK, dA, t);
-            int hits = 0;
-            for (int o0 = 0; o0 < Lt; o0 += 32 * kSupILP) {
-                int cc[kSupILP];
-#pragma unroll
-                for (int r = 0; r < kSupILP; ++r) {
-                    const int o = o0 + 32 * r + lane;
-                    cc[r] = o < Lt ? __ldg(G.adj + qt + o) : -1;
-                }
-#pragma unroll
-                for (int r = 0; r < kSupILP; ++r) {
-                    bool hit = false;
-                    if (cc[r] >= 0) {
-                        uint32_t h = ((uint32_t)cc[r] * 0x9E3779B1u) >> (32 - hbits);
-                        int y;
-                        while ((y = key[h]) != cc[r] && y != -1) h = (h + 1) & hm;
-                        if (y == cc[r]) {
-                            hit = true;
-                            atomicAdd(&cb[kpos[h]], 1);
-                            atomicAdd(sup + (qt + o0 + 32 * r + lane - dt), 1);
-                        }
-                    }
-                    hits += __popc(__ballot_sync(FULLMASK, hit));
-                }
-            }
-            const int et = __shfl_sync(FULLMASK, e, t);
-            if (lane == 0 && hits) atomicAdd(sup + et, hits);
-        }
-    }
-}
-
-template <int CAPT, bool STR = (CAPT > FSGC_SUP_CAPW), int NW = (STR ? 4 : 8)>
-__global__ void __launch_bounds__(NW * 32, 1) support_hash_kernel(
-    GraphDev G, OrientDev O, const int32_t* __restrict__ rev, const uint64_t* __restrict__ units, int64_t nunits,
-    int* __restrict__ sup, unsigned long long* queue, int shard, int nshards) {
-    typedef SupLayout<CAPT, STR, NW> Lay;
-    extern __shared__ __align__(16) unsigned char s_sup[];
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    unsigned char* tb = s_sup + w * Lay::warp_bytes;
-    int32_t* key = reinterpret_cast<int32_t*>(tb);
-    int16_t* kpos = reinterpret_cast<int16_t*>(tb + (size_t)Lay::HS * 4);
-    int32_t* cb = reinterpret_cast<int32_t*>(tb + (size_t)Lay::HS * 6);
-    unsigned char* wb = tb + Lay::table_bytes;
-    int32_t* pre = reinterpret_cast<int32_t*>(wb);
-    uint32_t* q0 = reinterpret_cast<uint32_t*>(wb + (FSGC_SUP_SEG + 4) * 4);
-    uint32_t* da = q0 + FSGC_SUP_SEG;
-    int32_t* ea = reinterpret_cast<int32_t*>(da + FSGC_SUP_SEG);
-    int32_t* cab = ea + FSGC_SUP_SEG;
-    int prev_b = -1, ob = 0, hbits = 5;
-    int64_t sb = 0;
-    const int64_t mine = nunits > shard ? (nunits - shard + nshards - 1) / nshards : 0;
-    for (;;) {
-        unsigned long long jq = 0;
-        if (lane == 0) jq = atomicAdd(queue, 1ull);
-        jq = __shfl_sync(FULLMASK, jq, 0);
-        if ((int64_t)jq >= mine) break;
-        // large tables: the largest middles (end of the degree order) first
-        const int64_t t = (int64_t)jq * nshards + shard;
-        const uint64_t un = __ldg(units + (Lay::STREAM ? nunits - 1 - t : t));
-        const int b = (int)(un >> 32), k = (int)(un & 0xffffffffu);
-        if (b != prev_b) {                    // (re)build the table of N+(b)
-            if (prev_b >= 0) {                // flush c(b', x) of the previous b'
-                const int64_t base = __ldg(O.oofs + prev_b);
-                for (int i = lane; i < ob; i += 32)
-                    if (cb[i]) atomicAdd(sup + base + i, cb[i]);
-            }
-            sb = __ldg(O.split + b);
-            ob = (int)(__ldg(G.offs + b + 1) - sb);
-            hbits = 5;
-            while ((1 << hbits) < 2 * ob) ++hbits;
-            __syncwarp();
-            for (int i = lane; i < (1 << hbits); i += 32) key[i] = -1;
-            for (int i = lane; i < ob; i += 32) cb[i] = 0;
-            __syncwarp();
-            const uint32_t hm = (1u << hbits) - 1;
-            for (int i = lane; i < ob; i += 32) {
-                const int x = __ldg(G.adj + sb + i);
-                uint32_t h = ((uint32_t)x * 0x9E3779B1u) >> (32 - hbits);
-                while (atomicCAS(&key[h], -1, x) != -1) h = (h + 1) & hm;
-                kpos[h] = (int16_t)i;
-            }
-            prev_b = b;
-            __syncwarp();
-        }
-        const int64_t ib0 = __ldg(G.offs + b) + (int64_t)k * FSGC_SUP_SEG;
-        const int len = (int)min((int64_t)FSGC_SUP_SEG, sb - ib0);
-        const int64_t rbase = ib0 - __ldg(O.oofs + b);
-        if (Lay::STREAM)
-            sup_slice_stream(G, O, rev, sup, ib0, len, rbase, key, kpos, cb, hbits, lane);
-        else
-            sup_slice(G, O, rev, sup, ib0, len, rbase, key, kpos, cb, hbits, pre, q0, da, ea, cab, lane);
-        __syncwarp();
-    }
-    if (prev_b >= 0) {
-        __syncwarp();
-        const int64_t base = __ldg(O.oofs + prev_b);
-        for (int i = lane; i < ob; i += 32)
-            if (cb[i]) atomicAdd(sup + base + i, cb[i]);
-    }
-}
-
 // One program of the Sec. 3.1 closed form, out of line: the kernels are short
 // and latency-bound, so a compact hot path (instruction-cache footprint)
 // matters more than call overhead.  `small`: the 64-bit bound holds.
@@ -796,8 +554,8 @@ __device__ __forceinline__ void edge_terms_eval(uint64_t nu, uint64_t nv, uint64
 }
 
 template <int NP>
-__global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, const CoreProg P, WorkDesc W,
-                                                      const int* __restrict__ sup, const EdgeTerms T,
+__global__ void __launch_bounds__(256) edge_fc_kernel(GraphDev G, OrientDev O, const __grid_constant__ CoreProg P, WorkDesc W,
+                                                      const int* __restrict__ sup, const __grid_constant__ EdgeTerms T,
                                                       const Sink S) {
     extern __shared__ u128 s_rows[];                 // [row entry][thread] (table path)
     // program table (checked fallback path): k | l << 8 | m << 16 | pattern << 24
@@ -939,6 +697,22 @@ struct VTerm {
     uint8_t pat, nz;
     uint8_t off[kMaxVennNz];     // row entries (base[r] + s_r - 1) of the regions with s_r > 0
 };
+// Z-term table (triangle cores whose every program is a single fringe type
+// or has all k = 1): fc from the intersection sizes Z[A] = |cap_{x in A} e(x)|
+// of the core-position sets A -- for a triangle core Z[{x}] = deg(x) - 2,
+// Z[{x,y}] = c(xy) - 1, Z[{u,v,w}] = t -- instead of the Venn diagram:
+//   single type (A, k):   fc = C(Z[A], k)
+//   all k = 1:            fc = sum_pi coef(pi) prod_B Z[A_B]  (partition
+//                         lattice, Moebius inversion -- PartTerm)
+// A term: signed coefficient x product of row entries C(Z[cm], j); terms of
+// the same pattern and the same factors are merged across programs.
+constexpr int kMaxZTerms = 512;
+struct ZTerm {
+    int64_t coef;
+    uint8_t pat, nf;
+    uint8_t f[6];                // row entries: zbase[cm] + j - 1
+};
+
 struct VennDev {
     const VTerm* __restrict__ terms;
     int32_t n;                   // terms; 0: table off (per-program Listing 5)
@@ -947,6 +721,14 @@ struct VennDev {
     int32_t warp;                // 1: one diagram per warp (large tables), 0: one per lane
     uint8_t maxs[64];            // per region: max s_r (0: no row)
     uint8_t base[64];            // per region: first row entry
+    // Z-term table (triangle cores; zn == 0: off)
+    const ZTerm* __restrict__ zterms;
+    int32_t zn;
+    int32_t znrows;
+    int32_t zneed7;              // some factor uses Z[{u,v,w}] = t
+    int32_t zk;                  // max fringes of one program (bound)
+    uint8_t zmaxj[8];            // per core mask cm: max j of C(Z[cm], j)
+    uint8_t zbase[8];            // per core mask cm: first row entry
 };
 
 // log2 upper bound of one pattern's fc sum on this diagram:
@@ -1164,227 +946,11 @@ __device__ __forceinline__ bool member(const GraphDev& G, const HubDev& H, int y
     return contains(G.adj + b, (int)(__ldg(G.offs + y + 1) - b), x);
 }
 
-constexpr int kTriWarps = 8;
+constexpr int kTriWarps = 8;   // warps per block of the triangle-core kernels
 constexpr int kTriLight = 32;     // N(u) longer than this: warp-cooperative triple intersection
 constexpr int kTriStack = 32;
 
-template <int NP>
-__global__ void __launch_bounds__(kTriWarps * 32) tri_core_kernel(GraphDev G, OrientDev O, HubDev H,
-                                                                   const CoreProg P, WorkDesc W,
-                                                                   const int* __restrict__ sup, const VennDev VD,
-                                                                   const Sink S) {
-    extern __shared__ u128 s_rows[];                     // small tables: rows [entry][thread]
-    __shared__ u128 s_vrows[kTriWarps][kMaxVennRows];   // large tables: rows per warp
-    __shared__ uint32_t s_leaf[kTriWarps][64][6];   // u, v, w, e(uv), e(uw), e(vw)
-    __shared__ uint32_t s_venn[kTriWarps][64][8];   // Venn over the q anchors
-    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
-    AccN<NP> acc;
-    acc.init();
-    unsigned long long nmatch = 0;
-    const int q = P.q, V = 1 << q, nprog = P.nprog;
-    // position mask F (bit0 u, bit1 v, bit2 w) -> Venn bit mask over the anchors
-    int proj[8];
-#pragma unroll
-    for (int F = 0; F < 8; ++F) {
-        int M = 0;
-        for (int b = 0; b < q; ++b)
-            if ((F >> P.anchor_pos[b]) & 1) M |= 1 << b;
-        proj[F] = M;
-    }
-    // t enters region F with sign +1 (|F| odd) or -1 (|F| = 2); the Venn over
-    // the anchors needs t only if some anchor region collects a nonzero sum of
-    // those signs (only when all three core vertices are anchors)
-    bool need_t = false;
-    {
-        int tco[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-#pragma unroll
-        for (int F = 1; F < 8; ++F) tco[proj[F]] += (__popc(F) & 1) ? 1 : -1;
-#pragma unroll
-        for (int M = 1; M < 8; ++M) need_t |= tco[M] != 0;
-    }
-    // this shard's roots, transposed over the grid (see edge_fc_kernel)
-    const int64_t total = W.end - W.begin;
-    const int64_t nchunks = (total + 31) / 32;
-    const int64_t mychunks = nchunks > W.shard ? (nchunks - W.shard + W.nshards - 1) / W.nshards : 0;
-    const int64_t nloc = mychunks * 32;
-    const int64_t nthreads = (int64_t)gridDim.x * blockDim.x;
-    const int64_t warp = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
-    const int64_t tpos = (int64_t)lane * (nthreads >> 5) + warp;
-
-    int64_t kq = 0;                  // this lane's next root slot
-    bool have = false, done = false;
-    int u = 0, v = 0;
-    int64_t e = 0, pa = 0, ea = 0, pb = 0, eb = 0, su = 0, sv = 0;
-    int cnt = 0;                     // leaves in the warp buffer (warp-uniform)
-
-    auto flush = [&]() {
-        __syncwarp();
-        // (1) triple intersections + Venn, one leaf per lane (two passes if > 32)
-        for (int base = 0; base < cnt; base += 32) {
-            const int li = base + lane;
-            const bool mine = li < cnt;
-            int lu = 0, lv = 0, lw = 0, du = 0, dv = 0, dw = 0, t = 0;
-            int cuv = 0, cuw = 0, cvw = 0;
-            if (mine) {
-                lu = (int)s_leaf[wib][li][0]; lv = (int)s_leaf[wib][li][1]; lw = (int)s_leaf[wib][li][2];
-                cuv = __ldg(sup + s_leaf[wib][li][3]);
-                cuw = __ldg(sup + s_leaf[wib][li][4]);
-                cvw = __ldg(sup + s_leaf[wib][li][5]);
-                du = (int)(__ldg(G.offs + lu + 1) - __ldg(G.offs + lu));
-                dv = (int)(__ldg(G.offs + lv + 1) - __ldg(G.offs + lv));
-                dw = (int)(__ldg(G.offs + lw + 1) - __ldg(G.offs + lw));
-            }
-            const bool heavy = mine && need_t && du > kTriLight;
-            if (mine && need_t && !heavy) {
-                Cursor cv, cw;
-                cv.init(G, H, lv);
-                cw.init(G, H, lw);
-                const int64_t b0 = __ldg(G.offs + lu);
-                for (int i = 0; i < du; ++i) {
-                    const int x = __ldg(G.adj + b0 + i);
-                    if (cv.has(x) && cw.has(x)) ++t;
-                }
-            }
-            unsigned hb = __ballot_sync(FULLMASK, heavy);
-            while (hb) {
-                const int who = __ffs(hb) - 1;
-                hb &= hb - 1;
-                const int hu = __shfl_sync(FULLMASK, lu, who), hv = __shfl_sync(FULLMASK, lv, who);
-                const int hw = __shfl_sync(FULLMASK, lw, who), hd = __shfl_sync(FULLMASK, du, who);
-                const int64_t b0 = __ldg(G.offs + hu);
-                int tt = 0;
-                for (int s0 = 0; s0 < hd; s0 += 32) {
-                    bool hit = false;
-                    if (s0 + lane < hd) {
-                        const int x = __ldg(G.adj + b0 + s0 + lane);
-                        hit = member(G, H, hv, x) && member(G, H, hw, x);
-                    }
-                    tt += __popc(__ballot_sync(FULLMASK, hit));
-                }
-                if (lane == who) t = tt;
-            }
-            if (mine) {
-                int R[8];
-                R[7] = t;
-                R[3] = cuv - 1 - t;
-                R[5] = cuw - 1 - t;
-                R[6] = cvw - 1 - t;
-                R[1] = du - 2 - R[3] - R[5] - t;
-                R[2] = dv - 2 - R[3] - R[6] - t;
-                R[4] = dw - 2 - R[5] - R[6] - t;
-                uint32_t vq[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-#pragma unroll
-                for (int F = 1; F < 8; ++F)
-                    if (proj[F]) vq[proj[F]] += (uint32_t)R[F];
-                for (int k = 0; k < V; ++k) s_venn[wib][li][k] = vq[k];
-            }
-        }
-        __syncwarp();
-        if (VD.n) {
-            if (VD.warp) {   // (2) fc by the Venn term table, one leaf at a time per warp
-                for (int li = 0; li < cnt; ++li) {
-                    uint32_t vloc[8];
-                    for (int k = 0; k < V; ++k) vloc[k] = s_venn[wib][li][k];
-                    venn_fc_warp<kTriStack>(vloc, q, P, VD, s_vrows[wib], lane, acc);
-                }
-            } else {         // (2) small tables: one leaf per lane, rows per thread
-                for (int base = 0; base < cnt; base += 32) {
-                    const int li = base + lane;
-                    const bool mine = li < cnt;
-                    uint32_t vloc[8];
-                    float bnd = 0.f;
-                    if (mine) {
-                        for (int k = 0; k < V; ++k) vloc[k] = s_venn[wib][li][k];
-                        bnd = venn_bound_log2(vloc, q, P) + VD.slack;
-                    }
-                    const bool all64 = __all_sync(FULLMASK, !mine || bnd < 55.f);
-                    if (mine && all64) {
-                        venn_terms_eval<uint64_t>(vloc, V, VD, (uint64_t*)(s_rows + threadIdx.x), 2 * blockDim.x, acc);
-                    } else if (mine && bnd < 119.f) {
-                        venn_terms_eval<u128>(vloc, V, VD, s_rows + threadIdx.x, blockDim.x, acc);
-                    } else if (mine) {                     // checked Listing 5 per program
-                        for (int pi = 0; pi < nprog; ++pi) {
-                            const FringeProg fp = P.prog[pi];
-                            bool o = false;
-                            const u128 f = fc_dispatch<kTriStack>(vloc, q, fp, o);
-                            acc.add(fp.pat, f, o);
-                        }
-                    }
-                }
-            }
-        } else {
-            // (2) fc over (leaf, program) pairs
-            const int pairs = cnt * nprog;
-            for (int tpair = lane; tpair < pairs; tpair += 32) {
-                const int li = tpair / nprog, pi = tpair - li * nprog;
-                uint32_t vloc[8];
-                for (int k = 0; k < V; ++k) vloc[k] = s_venn[wib][li][k];
-                const FringeProg fp = P.prog[pi];
-                bool o = false;
-                const u128 f = fc_dispatch<kTriStack>(vloc, q, fp, o);
-                acc.add(fp.pat, f, o);
-            }
-        }
-        nmatch += (lane == 0) ? (unsigned long long)cnt : 0ull;
-        cnt = 0;
-        __syncwarp();
-    };
-
-    for (;;) {
-        // refill: the next root of this lane that passes the degree filter
-        while (!have && !done) {
-            const int64_t L = kq * nthreads + tpos;
-            ++kq;
-            if (L >= nloc) { done = true; break; }
-            const int64_t tt = ((L >> 5) * W.nshards + W.shard) * 32 + (L & 31);
-            if (tt >= total) continue;
-            e = W.begin + tt;
-            u = __ldg(G.osrc + e);
-            v = __ldg(G.odst + e);
-            const int64_t ou = __ldg(G.offs + u), ou1 = __ldg(G.offs + u + 1);
-            const int64_t ov = __ldg(G.offs + v), ov1 = __ldg(G.offs + v + 1);
-            if (W.degfilter && ((int)(ou1 - ou) < P.mindeg[0] || (int)(ov1 - ov) < P.mindeg[1])) continue;
-            if (__ldg(sup + e) == 0) continue;       // no triangle on (u, v) at all
-            // w > v: the merge starts in N+(u) right after v (v's position
-            // in N+(u) is e's oriented offset)
-            su = __ldg(O.split + u); pa = su + (e - __ldg(O.oofs + u)) + 1; ea = ou1;
-            sv = __ldg(O.split + v); pb = sv; eb = ov1;
-            have = true;
-        }
-        if (__ballot_sync(FULLMASK, have) == 0) break;   // all lanes exhausted
-        // advance this lane's merge to its next triangle
-        bool found = false;
-        int w = 0;
-        int64_t fa = 0, fb = 0;
-        if (have) {
-            int x = pa < ea ? __ldg(G.adj + pa) : 0, y = pb < eb ? __ldg(G.adj + pb) : 0;
-            while (pa < ea && pb < eb) {
-                if (x < y) { if (++pa < ea) x = __ldg(G.adj + pa); }
-                else if (x > y) { if (++pb < eb) y = __ldg(G.adj + pb); }
-                else { found = true; w = x; fa = pa; fb = pb; ++pa; ++pb; break; }
-            }
-            if (!found) have = false;
-            if (found && W.degfilter) {
-                const int dw = (int)(__ldg(G.offs + w + 1) - __ldg(G.offs + w));
-                if (dw < P.mindeg[2]) found = false;
-            }
-        }
-        const unsigned fm = __ballot_sync(FULLMASK, found);
-        if (found) {
-            const int slot = cnt + __popc(fm & ((1u << lane) - 1));
-            s_leaf[wib][slot][0] = (uint32_t)u;
-            s_leaf[wib][slot][1] = (uint32_t)v;
-            s_leaf[wib][slot][2] = (uint32_t)w;
-            s_leaf[wib][slot][3] = (uint32_t)e;
-            s_leaf[wib][slot][4] = (uint32_t)(__ldg(O.oofs + u) + (fa - su));
-            s_leaf[wib][slot][5] = (uint32_t)(__ldg(O.oofs + v) + (fb - sv));
-        }
-        cnt += __popc(fm);
-        if (cnt >= 32) flush();
-    }
-    if (cnt) flush();
-    block_publish<NP>(acc, nmatch, S);
-}
+#include "listing.cuh"
 
 // ------------------------------------------------------------------------
 // General cores (p >= 3): one warp per root edge (atomic chunk queue, heavy
@@ -1464,9 +1030,9 @@ __device__ __noinline__ bool fc_partition(const uint32_t* venn, int q, const Par
 
 template <int NP>
 __global__ void __launch_bounds__(kCoreWarps * 32) core_kernel(GraphDev G, OrientDev O, HubDev H,
-                                                                const CoreProg P, WorkDesc W,
+                                                                const __grid_constant__ CoreProg P, WorkDesc W,
                                                                 const int* __restrict__ sup, TermDev TD,
-                                                                const VennDev VD, const Sink S,
+                                                                const __grid_constant__ VennDev VD, const Sink S,
                                                                 unsigned long long* queue) {
     extern __shared__ uint32_t smem[];
     __shared__ u128 s_vrows[kCoreWarps][kMaxVennRows];   // Venn-table binomial rows, per warp
@@ -1788,40 +1354,6 @@ int tune(const char* name, int dflt) {
     return r;
 }
 
-// the large-table support kernel (FSGC_SUP_BIG variant, see SupLayout), its
-// warps per block and dynamic shared memory
-const void* big_support_kernel(int* warps, size_t* bytes, int cap) {
-    if (cap == 4096) {
-        typedef SupLayout<4096, true, 1> L;
-        *warps = L::WARPS;
-        if (bytes) *bytes = L::bytes;
-        return (const void*)support_hash_kernel<4096, true, 1>;
-    }
-    if (cap == 2048) {
-        typedef SupLayout<2048, true, 2> L;
-        *warps = L::WARPS;
-        if (bytes) *bytes = L::bytes;
-        return (const void*)support_hash_kernel<2048, true, 2>;
-    }
-    const int mode = tune("FSGC_SUP_BIG", 0);
-    if (mode == 1) {
-        typedef SupLayout<FSGC_SUP_CAP, false, 4> L;
-        *warps = L::WARPS;
-        if (bytes) *bytes = L::bytes;
-        return (const void*)support_hash_kernel<FSGC_SUP_CAP, false, 4>;
-    }
-    if (mode == 2) {
-        typedef SupLayout<FSGC_SUP_CAP, true, 2> L;
-        *warps = L::WARPS;
-        if (bytes) *bytes = L::bytes;
-        return (const void*)support_hash_kernel<FSGC_SUP_CAP, true, 2>;
-    }
-    typedef SupLayout<FSGC_SUP_CAP> L;
-    *warps = L::WARPS;
-    if (bytes) *bytes = L::bytes;
-    return (const void*)support_hash_kernel<FSGC_SUP_CAP>;
-}
-
 // resident blocks per SM of a kernel on the current device (cached per
 // device / function / block / smem); raises the kernel's dynamic shared
 // memory opt-in on that device first (cudaFuncSetAttribute is per device).
@@ -1861,7 +1393,8 @@ struct Kernels {
     static const void* vertex() { return (const void*)vertex_core_kernel<NP>; }
     static const void* edge() { return (const void*)edge_fc_kernel<NP>; }
     static const void* core() { return (const void*)core_kernel<NP>; }
-    static const void* tri() { return (const void*)tri_core_kernel<NP>; }
+    static const void* tri() { return (const void*)list_warp_kernel<true, NP>; }
+    static const void* tri_block() { return (const void*)list_block_kernel<true, NP>; }
 };
 
 // smallest NP in {1,2,4,8,16} holding npats
@@ -1873,6 +1406,24 @@ const void* kernel_for(int kind, int np) {
     switch (np) { FSGC_K(1) FSGC_K(2) FSGC_K(4) FSGC_K(8) FSGC_K(16) }
 #undef FSGC_K
     return nullptr;
+}
+
+// the block-table triangle-core kernel of accumulator class np
+const void* tri_block_kernel(int np) {
+    switch (np) {
+        case 1: return Kernels<1>::tri_block();
+        case 2: return Kernels<2>::tri_block();
+        case 4: return Kernels<4>::tri_block();
+        case 8: return Kernels<8>::tri_block();
+        default: return Kernels<16>::tri_block();
+    }
+}
+
+// hash bits of a block table holding out-degree `maxout` at load <= 1/2
+int table_hbits(int64_t maxout) {
+    int hb = 5;
+    while ((1ll << hb) < 2 * maxout) ++hb;
+    return hb;
 }
 
 }  // namespace
@@ -2011,6 +1562,9 @@ struct PassExec {
     size_t smem_fc = 0;        // dynamic shared memory of edge_fc_kernel
     VennDev vd{};              // triangle / general cores: the Venn term table (vd.n == 0: off)
     size_t smem_vd = 0;        // its per-thread binomial rows (dynamic shared memory)
+    int64_t grid2 = 0;         // triangle cores: the block-table launch ...
+    size_t smem2 = 0;          // ... its shared memory
+    int hbits2 = 5;            // ... and table hash bits
 };
 
 // the term table of an edge-core pass (see EdgeTerms); et.n = 0 when a
@@ -2131,6 +1685,72 @@ static bool build_venn_terms(const CoreProg& cp, std::vector<VTerm>* out, VennDe
     hd->slack = std::log2((float)mp) + 2.f;
     return true;
 }
+// the Z-term table of a triangle-core pass (see ZTerm): false when some
+// program is neither a single fringe type nor all-k = 1, or past the limits
+static bool build_z_terms(const CoreProg& cp, const std::vector<std::vector<PartTerm>>& pterms,
+                          std::vector<ZTerm>* out, VennDev* hd) {
+    out->clear();
+    if (cp.p != 3) return false;
+    auto cmask = [&](int venn_mask) {
+        int cm = 0;
+        for (int b = 0; b < cp.q; ++b)
+            if ((venn_mask >> b) & 1) cm |= 1 << cp.anchor_pos[b];
+        return cm;
+    };
+    // (pattern, sorted factor list (cm << 8 | j)) -> coefficient
+    std::map<std::pair<int, std::vector<int>>, int64_t> acc;
+    int maxj[8] = {0}, zk = 0;
+    for (int pi = 0; pi < cp.nprog; ++pi) {
+        const FringeProg& fp = cp.prog[pi];
+        zk = std::max(zk, (int)fp.ksum);
+        if (fp.s == 0) {
+            acc[std::make_pair((int)fp.pat, std::vector<int>())] += 1;
+        } else if (fp.s == 1) {
+            const int cm = cmask(fp.anch[0]), j = fp.k[0];
+            if (j > 63) return false;
+            maxj[cm] = std::max(maxj[cm], j);
+            acc[std::make_pair((int)fp.pat, std::vector<int>{cm << 8 | j})] += 1;
+        } else {
+            if (pterms[pi].empty()) return false;
+            for (const PartTerm& tm : pterms[pi]) {
+                std::vector<int> f;
+                for (int b = 0; b < tm.nb; ++b) {
+                    const int cm = cmask(tm.mask[b]);
+                    maxj[cm] = std::max(maxj[cm], 1);
+                    f.push_back(cm << 8 | 1);
+                }
+                std::sort(f.begin(), f.end());
+                acc[std::make_pair((int)fp.pat, f)] += tm.coef;
+            }
+        }
+    }
+    int nrows = 0;
+    for (int cm = 1; cm < 8; ++cm) {
+        hd->zmaxj[cm] = (uint8_t)maxj[cm];
+        hd->zbase[cm] = (uint8_t)nrows;
+        nrows += maxj[cm];
+    }
+    hd->zmaxj[0] = 0;
+    for (auto& kv : acc) {
+        if (kv.second == 0) continue;
+        if (kv.first.second.size() > 6) return false;
+        ZTerm t;
+        std::memset(&t, 0, sizeof t);
+        t.coef = kv.second;
+        t.pat = (uint8_t)kv.first.first;
+        for (int f : kv.first.second) t.f[t.nf++] = (uint8_t)(hd->zbase[f >> 8] + (f & 255) - 1);
+        out->push_back(t);
+    }
+    if (out->empty() || (int)out->size() > kMaxZTerms || nrows > kMaxVennRows) return false;
+    int progs_per_pat[FSGC_MAXPATS] = {0}, mp = 1;
+    for (int pi = 0; pi < cp.nprog; ++pi) mp = std::max(mp, ++progs_per_pat[cp.prog[pi].pat]);
+    hd->slack = std::log2((float)mp) + 2.f;
+    hd->zn = (int32_t)out->size();
+    hd->znrows = nrows;
+    hd->zneed7 = maxj[7] > 0;
+    hd->zk = zk;
+    return true;
+}
 }  // namespace
 
 // device copies of the partition-lattice term tables of a pattern batch;
@@ -2141,12 +1761,14 @@ struct DevTerms {
     int32_t* off = nullptr;
     int32_t* cnt = nullptr;
     VTerm* vterms = nullptr;        // Venn term tables of all passes
+    ZTerm* zterms = nullptr;        // Z-term tables of all passes
     std::vector<VennDev> vhdr;      // per pass (terms point into vterms)
     ~DevTerms() {
         if (terms) cudaFree(terms);
         if (off) cudaFree(off);
         if (cnt) cudaFree(cnt);
         if (vterms) cudaFree(vterms);
+        if (zterms) cudaFree(zterms);
     }
 };
 
@@ -2161,9 +1783,11 @@ struct fsgc_plan {
     // reads it (edge, triangle and general cores), at ws[sup_off, + 4 m)
     int sup_first = -1;            // first pass reading it (-1: none)
     size_t sup_off = 0;            // the array; its work-queue counter 256 bytes before
-    int64_t grid_sup = 1;          // merge part (heavy middle vertices)
-    int64_t grid_hash = 1;         // wedge-hash part, warp tables
-    int64_t grid_hash_big = 1;     // wedge-hash part, block tables
+    int64_t grid_sup = 1;          // merge kernel (small graphs / FSGC_SUP_MERGE_ONLY)
+    int64_t grid_hash = 1;         // listing kernel, warp tables
+    int64_t grid_hash_big = 1;     // listing kernel, block tables
+    int hbits_big = 5;             // block tables: hash bits ...
+    size_t smem_big = 0;           // ... and shared memory
     int sup_shard = 0, sup_nshards = 1;   // FSGC_FLAG_SHARD_SUPPORT: this shard's part
     std::vector<cudaEvent_t> ev;   // support begin/end, then begin/end per pass
     unsigned long long* trace = nullptr;
@@ -2214,8 +1838,12 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
         X.W = WorkDesc{b, e, opts.shard_index, opts.shard_count, 4,
                        (opts.flags & FSGC_FLAG_NO_DEGREE_FILTER) ? 0 : 1, nullptr};
         X.kind = cp.root_mode == ROOT_VERTEX ? 0 : (cp.p == 2 ? 1 : 2);
+        // triangle cores with full symmetry breaking (u < v < w) over the
+        // whole root range: the listing kernels (listing.cuh) enumerate them
+        // by middle vertex; partial root ranges go to the generic kernel
+        const bool whole_range = opts.root_begin <= 0 && opts.root_end < 0;
         if (X.kind == 2 && cp.p == 3 && cp.back[2] == 3 && cp.root_mode == ROOT_ORIENTED && (cp.gt[2] & 2) &&
-            !tune("FSGC_NO_TRI", 0)) {
+            (cp.gt[2] & 1) && (cp.gt[1] & 1) && whole_range && !tune("FSGC_NO_TRI", 0)) {
             bool fits = true;   // Listing 5 stack bound of the triangle kernel
             for (int k = 0; k < cp.nprog; ++k) fits = fits && cp.prog[k].depth <= kTriStack;
             if (fits) X.kind = 3;
@@ -2235,10 +1863,9 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
                                                             (mine + 7) / 8));
             if (tune("FSGC_EDGE_BLOCKS", 0) > 0) X.grid = tune("FSGC_EDGE_BLOCKS", 0);
         } else if (X.kind == 3) {
-            int64_t mine = ((e - b) + 31) / 32;
-            mine = (mine + opts.shard_count - 1) / opts.shard_count;
-            X.grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy(kernel_for(3, X.npc), kTriWarps * 32, 0),
-                                                            (mine + kTriWarps - 1) / kTriWarps));
+            // grids and shared memory after the Venn tables (below); block
+            // partials for both launches
+            X.grid = (int64_t)nsm * 16;
         } else {
             X.smem = (size_t)kCoreWarps * (32 * FSGC_MAXC + 32 * (1u << cp.q)) * sizeof(uint32_t);
             int64_t nchunks = ((e - b) + X.W.chunk - 1) / X.W.chunk;
@@ -2263,19 +1890,22 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
         off += X.bytes;
     }
     if (P->sup_first >= 0) {
-        P->grid_sup = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occupancy((const void*)support_kernel, 256, 0),
-                                                             (g->nsup_heavy + 255) / 256));
-        typedef SupLayout<FSGC_SUP_CAPW> LS;
-        P->grid_hash = std::max<int64_t>(1, std::min<int64_t>(
-            (int64_t)nsm * occupancy((const void*)support_hash_kernel<FSGC_SUP_CAPW>, LS::WARPS * 32, LS::bytes),
-            (g->nsup_units + LS::WARPS - 1) / LS::WARPS));
-        int warps_big = 0;
-        const void* fn_big = big_support_kernel(&warps_big, nullptr, g->sup_cap_big);
-        size_t bytes_big = 0;
-        big_support_kernel(&warps_big, &bytes_big, g->sup_cap_big);
-        P->grid_hash_big = std::max<int64_t>(1, std::min<int64_t>(
-            (int64_t)nsm * occupancy(fn_big, warps_big * 32, bytes_big),
-            (g->nsup_units_big + warps_big - 1) / warps_big));
+        if (g->sup_hash) {
+            typedef WarpTabLayout<false> LS;
+            P->grid_hash = std::max<int64_t>(1, std::min<int64_t>(
+                (int64_t)nsm * occupancy((const void*)list_warp_kernel<false, 1>, kWarpTabWarps * 32, LS::bytes),
+                (g->nsup_units + kWarpTabWarps - 1) / kWarpTabWarps));
+            P->hbits_big = table_hbits(g->sup_maxout);
+            P->smem_big = blocktab_table_bytes(1 << P->hbits_big, (int)g->sup_maxout, false);
+            const int occ = occupancy((const void*)list_block_kernel<false, 1>, kBlockTabWarps * 32, P->smem_big);
+            if (g->nsup_units_big > 0 && occ == 0)
+                FSGC_FAIL(FSGC_ERR_INVALID, "block table of out-degree %lld does not fit shared memory",
+                          (long long)g->sup_maxout);
+            P->grid_hash_big = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * occ, g->nsup_units_big));
+        }
+        if (g->nsup_merge > 0)
+            P->grid_sup = std::max<int64_t>(1, std::min<int64_t>(
+                (int64_t)nsm * occupancy((const void*)support_kernel, 256, 0), (g->nsup_merge + 255) / 256));
         if ((opts.flags & FSGC_FLAG_SHARD_SUPPORT) && opts.shard_count > 1) {
             P->sup_shard = opts.shard_index;
             P->sup_nshards = opts.shard_count;
@@ -2315,6 +1945,8 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
             // Venn term tables (pattern-only, so cached with the rest)
             std::vector<VTerm> vall;
             std::vector<size_t> vbase;
+            std::vector<ZTerm> zall;
+            std::vector<size_t> zbase;
             for (auto& X : P->passes) {
                 VennDev hd;
                 std::memset(&hd, 0, sizeof hd);
@@ -2327,8 +1959,28 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
                     std::memset(&hd, 0, sizeof hd);
                     vbase.push_back(0);
                 }
+                // triangle cores: the Z-term table when every program allows it
+                std::vector<ZTerm> zt;
+                VennDev zh;
+                std::memset(&zh, 0, sizeof zh);
+                if (X.kind == 3 && !tune("FSGC_NO_Z_TERMS", 0) && build_z_terms(X.plan.prog, X.plan.terms, &zt, &zh)) {
+                    zbase.push_back(zall.size());
+                    zall.insert(zall.end(), zt.begin(), zt.end());
+                    hd.zn = zh.zn; hd.znrows = zh.znrows; hd.zneed7 = zh.zneed7; hd.zk = zh.zk;
+                    hd.slack = std::max(hd.slack, zh.slack);
+                    std::memcpy(hd.zmaxj, zh.zmaxj, 8);
+                    std::memcpy(hd.zbase, zh.zbase, 8);
+                } else {
+                    zbase.push_back(0);
+                }
                 T->vhdr.push_back(hd);
             }
+            if (!zall.empty()) {
+                FSGC_CUDA(cudaMalloc(&T->zterms, zall.size() * sizeof(ZTerm)));
+                FSGC_CUDA(cudaMemcpy(T->zterms, zall.data(), zall.size() * sizeof(ZTerm), cudaMemcpyHostToDevice));
+            }
+            for (size_t i = 0; i < T->vhdr.size(); ++i)
+                if (T->vhdr[i].zn) T->vhdr[i].zterms = T->zterms + zbase[i];
             if (!vall.empty()) {
                 FSGC_CUDA(cudaMalloc(&T->vterms, vall.size() * sizeof(VTerm)));
                 FSGC_CUDA(cudaMemcpy(T->vterms, vall.data(), vall.size() * sizeof(VTerm), cudaMemcpyHostToDevice));
@@ -2358,6 +2010,32 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
             if (tune("FSGC_VENN_INFO", 0))
                 fprintf(stderr, "[venn] pass kind %d: %d terms, %d rows, %s mode\n", X.kind, X.vd.n, X.vd.nrows,
                         X.vd.warp ? "warp" : "lane");
+        }
+        // triangle-core passes: the two listing launches (warp tables, block
+        // tables), persistent grids at full occupancy
+        for (auto& X : P->passes) {
+            if (X.kind != 3) continue;
+            // lane-mode term rows (kTriWarps * 32 threads): Venn table and/or Z table
+            const size_t rows = std::max(X.smem_vd, X.vd.zn ? (size_t)X.vd.znrows * sizeof(u128) * kTriWarps * 32
+                                                              : (size_t)0);
+            X.smem = WarpTabLayout<true>::bytes + rows;
+            int occ = occupancy(kernel_for(3, X.npc), kWarpTabWarps * 32, X.smem);
+            if (occ == 0) FSGC_FAIL(FSGC_ERR_INVALID, "triangle-core pass: shared memory %zu B does not fit", X.smem);
+            const int64_t units_w = (g->nsup_units + opts.shard_count - 1) / opts.shard_count;
+            const int64_t units_b = (g->nsup_units_big + opts.shard_count - 1) / opts.shard_count;
+            X.grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * std::min(occ, 16),
+                                                            (units_w + kWarpTabWarps - 1) / kWarpTabWarps));
+            X.hbits2 = table_hbits(g->sup_maxout);
+            X.smem2 = blocktab_table_bytes(1 << X.hbits2, (int)g->sup_maxout, true) +
+                      kBlockTriWarps * blocktab_warp_bytes(true) + rows;
+            occ = occupancy(tri_block_kernel(X.npc), kBlockTriWarps * 32, X.smem2);
+            if (occ == 0 && units_b > 0)
+                FSGC_FAIL(FSGC_ERR_INVALID, "triangle-core pass: block table of out-degree %lld does not fit "
+                          "shared memory (%zu B)", (long long)g->sup_maxout, X.smem2);
+            X.grid2 = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * std::max(1, std::min(occ, 16)) ,
+                                                             std::max<int64_t>(1, units_b)));
+            if (X.grid + X.grid2 > (int64_t)nsm * 16)
+                FSGC_FAIL(FSGC_ERR_INTERNAL, "triangle-core pass: block partials overflow");
         }
     }
     P->ev.resize(2 + 2 * P->passes.size());
@@ -2411,32 +2089,35 @@ extern "C" int fsgc_plan_enqueue_stage(const fsgc_plan* P, void* workspace, void
         unsigned long long* dq = (unsigned long long*)((unsigned char*)dsup - 256);   // 2 queue counters
         unsigned long long* dq1 = dq + 1;
         FSGC_CUDA(cudaEventRecordWithFlags(P->ev[0], st, evflags));
-        // FSGC_SUP_MERGE_ONLY=1 (experiments): the merge kernel over every
-        // oriented edge (the work list holds the light ones after the heavy)
-        const bool merge_only = tune("FSGC_SUP_MERGE_ONLY", 0) != 0;
-        if (g->nsup_units_big > 0 && !merge_only) {
-            int nw = 0;
-            size_t nb = 0;
-            const void* fn = big_support_kernel(&nw, &nb, g->sup_cap_big);
-            void* args[] = {(void*)&G, (void*)&O, (void*)&g->rev, (void*)&g->sup_units_big, (void*)&g->nsup_units_big,
-                            (void*)&dsup, (void*)&dq1, (void*)&P->sup_shard, (void*)&P->sup_nshards};
-            FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)P->grid_hash_big), dim3(nw * 32), args, nb, st));
+        // listing kernels (graphs >= FSGC_SUP_HASH_MIN_M edges), else the
+        // merge kernel over every oriented edge (also FSGC_SUP_MERGE_ONLY=1:
+        // the independent check of the listing kernels)
+        const bool merge_only = g->nsup_merge > 0 && (!g->sup_hash || tune("FSGC_SUP_MERGE_ONLY", 0) != 0);
+        HubDev Hd{g->hub_base, g->hub_words, g->hub_bits};
+        const CoreProg* cp0 = &P->passes[P->sup_first].plan.prog;   // unused by the support visitor
+        WorkDesc W0{};
+        VennDev V0{};
+        Sink S0{};
+        if (!merge_only && g->nsup_units_big > 0) {
+            int hb = P->hbits_big, mo = (int)g->sup_maxout;
+            void* args[] = {(void*)&G, (void*)&O, (void*)&Hd, (void*)&g->rev, (void*)&g->sup_units_big,
+                            (void*)&g->nsup_units_big, (void*)&hb, (void*)&mo, (void*)&dsup, (void*)&dq1,
+                            (void*)&P->sup_shard, (void*)&P->sup_nshards, (void*)cp0, (void*)&W0, (void*)&V0,
+                            (void*)&S0};
+            FSGC_CUDA(cudaLaunchKernel((const void*)list_block_kernel<false, 1>, dim3((unsigned)P->grid_hash_big),
+                                       dim3(kBlockTabWarps * 32), args, P->smem_big, st));
         }
-        if (g->nsup_units > 0 && !merge_only) {
-            typedef SupLayout<FSGC_SUP_CAPW> LS;
-            support_hash_kernel<FSGC_SUP_CAPW><<<(int)P->grid_hash, LS::WARPS * 32, LS::bytes, st>>>(
-                G, O, g->rev, g->sup_units, g->nsup_units, dsup, dq, P->sup_shard, P->sup_nshards);
-            FSGC_CUDA(cudaGetLastError());
+        if (!merge_only && g->nsup_units > 0) {
+            void* args[] = {(void*)&G, (void*)&O, (void*)&Hd, (void*)&g->rev, (void*)&g->sup_units,
+                            (void*)&g->nsup_units, (void*)&dsup, (void*)&dq, (void*)&P->sup_shard,
+                            (void*)&P->sup_nshards, (void*)cp0, (void*)&W0, (void*)&V0, (void*)&S0};
+            FSGC_CUDA(cudaLaunchKernel((const void*)list_warp_kernel<false, 1>, dim3((unsigned)P->grid_hash),
+                                       dim3(kWarpTabWarps * 32), args, WarpTabLayout<false>::bytes, st));
         }
-        const int64_t nmerge = merge_only ? g->m : g->nsup_heavy;
-        if (nmerge > 0) {
-            const int grid = merge_only ? (int)std::max<int64_t>(P->grid_sup, std::min<int64_t>(
-                                              (int64_t)sm_count() * occupancy((const void*)support_kernel, 256, 0),
-                                              (g->m + 255) / 256))
-                                        : (int)P->grid_sup;
-            support_kernel<<<grid, 256, 0, st>>>(G, O, nmerge, dsup, g->sorder, g->ssrc,
-                                                              g->sdst, P->sup_shard, P->sup_nshards,
-                                                              P->trace ? P->trace + (1 << 17) : nullptr);
+        if (merge_only) {
+            support_kernel<<<(int)P->grid_sup, 256, 0, st>>>(G, O, g->nsup_merge, dsup, g->sorder, g->ssrc, g->sdst,
+                                                             P->sup_shard, P->sup_nshards,
+                                                             P->trace ? P->trace + (1 << 17) : nullptr);
             FSGC_CUDA(cudaGetLastError());
         }
         FSGC_CUDA(cudaEventRecordWithFlags(P->ev[1], st, evflags));
@@ -2461,14 +2142,33 @@ extern "C" int fsgc_plan_enqueue_stage(const fsgc_plan* P, void* workspace, void
             TermDev TD{P->terms->terms, P->terms->off + X.term_base, P->terms->cnt + X.term_base};
             void* args_c[] = {(void*)&G, (void*)&O, (void*)&Hd, (void*)&cp, (void*)&W, (void*)&dsup, (void*)&TD,
                               (void*)&X.vd, (void*)&S, (void*)&dqueue};
-            void* args_t[] = {(void*)&G, (void*)&O, (void*)&Hd, (void*)&cp, (void*)&W, (void*)&dsup, (void*)&X.vd,
-                              (void*)&S};
+            // triangle cores: two listing launches into one sink (one 128-bit
+            // atomic per block; the block launch's partials after the warp
+            // launch's), queues at dmatch[1], dmatch[2]
+            Sink St = S;
+            St.mode = 1;
+            Sink St2 = St;
+            St2.parts = St.parts + X.grid;
+            unsigned long long* dqueue2 = dmatch + 2;
+            int shard = W.shard, nsh = W.nshards, hb2 = X.hbits2, mo = (int)g->sup_maxout;
+            void* args_t[] = {(void*)&G, (void*)&O, (void*)&Hd, (void*)&g->rev, (void*)&g->sup_units,
+                              (void*)&g->nsup_units, (void*)&dsup, (void*)&dqueue, (void*)&shard, (void*)&nsh,
+                              (void*)&cp, (void*)&W, (void*)&X.vd, (void*)&St};
+            void* args_t2[] = {(void*)&G, (void*)&O, (void*)&Hd, (void*)&g->rev, (void*)&g->sup_units_big,
+                               (void*)&g->nsup_units_big, (void*)&hb2, (void*)&mo, (void*)&dsup, (void*)&dqueue2,
+                               (void*)&shard, (void*)&nsh, (void*)&cp, (void*)&W, (void*)&X.vd, (void*)&St2};
             if (X.kind == 0)
                 FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(256), args_v, 0, st));
             else if (X.kind == 1)    // (B) fringe counts per root edge
                 FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(256), args_e, X.smem_fc, st));
-            else if (X.kind == 3)
-                FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(kTriWarps * 32), args_t, X.smem_vd, st));
+            else if (X.kind == 3) {
+                if (g->nsup_units_big > 0)
+                    FSGC_CUDA(cudaLaunchKernel(tri_block_kernel(X.npc), dim3((unsigned)X.grid2),
+                                               dim3(kBlockTriWarps * 32), args_t2, X.smem2, st));
+                if (g->nsup_units > 0)
+                    FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(kWarpTabWarps * 32), args_t, X.smem,
+                                               st));
+            }
             else
                 FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(kCoreWarps * 32), args_c,
                                            X.smem + X.smem_vd, st));
@@ -2502,9 +2202,13 @@ extern "C" int fsgc_plan_decode(const fsgc_plan* P, const void* raw, fsgc_result
         if (sup_here && cudaEventElapsedTime(&ams, P->ev[0], P->ev[1]) != cudaSuccess) ams = -1.f;
         if (cudaEventElapsedTime(&kms, P->ev[2 + 2 * pi], P->ev[3 + 2 * pi]) != cudaSuccess) kms = -1.f;
         cudaGetLastError();   // timing is best effort (e.g. events recorded inside a graph)
-        const int launches = (X.W.end > X.W.begin ? 1 : 0) +
-                             (sup_here ? (P->g->nsup_units > 0 ? 1 : 0) + (P->g->nsup_units_big > 0 ? 1 : 0) +
-                                             (P->g->nsup_heavy > 0 ? 1 : 0) : 0);
+        const fsgc_graph* g = P->g;
+        const bool merge_only = g->nsup_merge > 0 && (!g->sup_hash || tune("FSGC_SUP_MERGE_ONLY", 0) != 0);
+        const int sup_launches = merge_only ? 1 : (g->nsup_units > 0 ? 1 : 0) + (g->nsup_units_big > 0 ? 1 : 0);
+        const int pass_launches = X.W.end <= X.W.begin ? 0
+                                  : X.kind == 3 ? (g->nsup_units > 0 ? 1 : 0) + (g->nsup_units_big > 0 ? 1 : 0)
+                                                : 1;
+        const int launches = pass_launches + (sup_here ? sup_launches : 0);
         for (size_t mi = 0; mi < X.plan.members.size(); ++mi) {
             fsgc_result& r = results[X.plan.members[mi]];
             r.raw.lo = acc[mi].lo;

@@ -145,26 +145,19 @@ struct UpperTri {
     __host__ __device__ bool operator()(const uint64_t& k) const { return (k >> B) < (k & mask); }
 };
 
-// merge-part work order: key = merge length out(u) + out(v) of oriented
-// edge i (capped) when its middle vertex v has out(v) > FSGC_SUP_CAP, else
-// the maximum key (sorted to the end, not used); value = i; sorted, so the 32
-// lanes of a warp get roots of similar cost (degree-aware binning, north_star)
+// merge-kernel work order: key = merge length out(u) + out(v) of oriented
+// edge i (capped at 2^20 - 1), value = i; sorted, so the 32 lanes of a warp
+// get roots of similar cost (degree-aware binning, north_star)
 __global__ void support_work_keys(const int64_t* __restrict__ offs, const int64_t* __restrict__ split,
                                   const int32_t* __restrict__ osrc, const int32_t* __restrict__ odst, int64_t m,
-                                  uint32_t* __restrict__ key, int32_t* __restrict__ idx,
-                                  unsigned long long* nheavy, int64_t cap) {
-    int cnt = 0;
+                                  uint32_t* __restrict__ key, int32_t* __restrict__ idx) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < m;
          i += (int64_t)gridDim.x * blockDim.x) {
         const int u = osrc[i], v = odst[i];
-        const int64_t ov = offs[v + 1] - split[v];
-        const int64_t w = (offs[u + 1] - split[u]) + ov;
-        const bool heavy = ov > cap;
-        key[i] = heavy ? (uint32_t)(w < (1 << 20) - 1 ? w : (1 << 20) - 2) : (uint32_t)((1 << 20) - 1);
+        const int64_t w = (offs[u + 1] - split[u]) + (offs[v + 1] - split[v]);
+        key[i] = (uint32_t)(w < (1 << 20) - 1 ? w : (1 << 20) - 1);
         idx[i] = (int32_t)i;
-        cnt += heavy;
     }
-    if (cnt) atomicAdd(nheavy, (unsigned long long)cnt);
 }
 
 // rev[i - oofs[b]] = oriented index of (a, b) for the in-entry a = adj[i] of
@@ -179,22 +172,29 @@ __global__ void rev_keys(const int32_t* __restrict__ osrc, const int32_t* __rest
     }
 }
 
-// wedge-hash units per middle vertex b (cnt[n] = 0 for the scans):
-// small-table units ceil(in(b) / SEG) when 1 <= out(b) <= CAPW, large-table
-// units ceil(in(b) / SEG) when CAPW < out(b) <= CAP
+// triangle-listing units per middle vertex b (cnt[n] = 0 for the scans):
+// warp-table units ceil(in(b) / SEG) when 1 <= out(b) <= capw, block-table
+// units ceil(in(b) / CHUNK) when out(b) > capw; maxout = max out(b) of a
+// block-table middle (sizes the block tables)
 __global__ void unit_counts(const int64_t* __restrict__ offs, const int64_t* __restrict__ split, int64_t n,
-                            int64_t* __restrict__ cnt, int64_t* __restrict__ cnt_big, int64_t cap) {
+                            int64_t* __restrict__ cnt, int64_t* __restrict__ cnt_big, int64_t capw,
+                            unsigned long long* maxout) {
+    unsigned long long mx = 0;
     for (int64_t b = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; b <= n;
          b += (int64_t)gridDim.x * blockDim.x) {
         int64_t c = 0, cb = 0;
         if (b < n) {
             const int64_t in = split[b] - offs[b], out = offs[b + 1] - split[b];
-            if (in >= 1 && out >= 1 && out <= FSGC_SUP_CAPW) c = (in + FSGC_SUP_SEG - 1) / FSGC_SUP_SEG;
-            if (in >= 1 && out > FSGC_SUP_CAPW && out <= cap) cb = (in + FSGC_SUP_SEG - 1) / FSGC_SUP_SEG;
+            if (in >= 1 && out >= 1 && out <= capw) c = (in + FSGC_SUP_SEG - 1) / FSGC_SUP_SEG;
+            if (in >= 1 && out > capw) {
+                cb = (in + FSGC_SUP_CHUNK - 1) / FSGC_SUP_CHUNK;
+                mx = mx > (unsigned long long)out ? mx : (unsigned long long)out;
+            }
         }
         cnt[b] = c;
         cnt_big[b] = cb;
     }
+    if (mx) atomicMax(maxout, mx);
 }
 
 __global__ void unit_fill(const int64_t* __restrict__ uofs, int64_t n, uint64_t* __restrict__ units) {
@@ -423,24 +423,27 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
         if (b > tmp_bytes) { FSGC_CUDA(tmp.alloc(b, st)); tmp_bytes = b; }
         FSGC_CUDA(cub::DeviceScan::ExclusiveSum(tmp.ptr, b, oofs.ptr, oofs.ptr, n + 1, st));
     }
-    // support pass, merge part: heavy-middle edges sorted by merge length
-    // with their (u, v) gathered; wedge-hash part: rev index + units
+    // Triangle listing from the middle vertex (support pass and triangle-core
+    // pass, count.cu): rev index + work units of the middles b, split at
+    // out(b) = capw into warp-table units (SEG in-entries) and block-table
+    // units (FSGC_SUP_CHUNK in-entries).  The merge-kernel work list (every
+    // oriented edge in merge-length order) only where the merge kernel runs:
+    // graphs below FSGC_SUP_HASH_MIN_M edges (launch-latency bound: the merge
+    // kernel alone is fastest there) or FSGC_SUP_MERGE_ONLY (the independent
+    // check of the hash kernels).
     DevBuf<int32_t> sorder, ssrc, sdst, rev;
     DevBuf<uint64_t> units, units_big;
     DevBuf<int64_t> ucnt, ucnt_big;
     FSGC_CUDA(cudaMemsetAsync(dnum.ptr, 0, 2 * sizeof(int64_t), st));
-    // small graphs (launch-latency bound): the merge part alone, over every
-    // edge (FSGC_SUP_HASH_MIN_M overrides the threshold)
     int64_t hash_min_m = 1 << 20;
     if (const char* v = getenv("FSGC_SUP_HASH_MIN_M")) hash_min_m = atoll(v);
     const bool use_hash = m >= hash_min_m;
-    // FSGC_SUP_CAP_BIG (experiments): large-table cap 1024 (default), 2048 or 4096
-    int64_t cap_big = FSGC_SUP_CAP;
-    if (const char* v = getenv("FSGC_SUP_CAP_BIG")) {
-        const int64_t c = atoll(v);
-        if (c == 2048 || c == 4096) cap_big = c;
-    }
-    if (m > 0 && use_hash) {
+    const bool merge_list = !use_hash || (getenv("FSGC_SUP_MERGE_ONLY") && atoi(getenv("FSGC_SUP_MERGE_ONLY")));
+    // FSGC_SUP_CAPW (tests): warp-table cap below the compiled 256, so small
+    // graphs reach the block-table kernels
+    int64_t capw = FSGC_SUP_CAPW;
+    if (const char* v = getenv("FSGC_SUP_CAPW")) capw = std::max<int64_t>(1, std::min<int64_t>(atoll(v), FSGC_SUP_CAPW));
+    if (m > 0) {
         {   // rev = oriented edge ids in (b, a) order = the in-entries' CSR order
             DevBuf<uint64_t> rk0, rk1;
             DevBuf<int32_t> rv1;
@@ -460,7 +463,8 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
         }
         FSGC_CUDA(ucnt.alloc(n + 1, st));
         FSGC_CUDA(ucnt_big.alloc(n + 1, st));
-        unit_counts<<<grid_for(n + 1), 256, 0, st>>>(offs.ptr, split.ptr, n, ucnt.ptr, ucnt_big.ptr, cap_big);
+        unit_counts<<<grid_for(n + 1), 256, 0, st>>>(offs.ptr, split.ptr, n, ucnt.ptr, ucnt_big.ptr, capw,
+                                                     (unsigned long long*)dnum.ptr + 1);
         FSGC_CUDA(cudaGetLastError());
         size_t b = 0;
         FSGC_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, b, ucnt.ptr, ucnt.ptr, n + 1, st));
@@ -468,22 +472,20 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
         FSGC_CUDA(cub::DeviceScan::ExclusiveSum(tmp.ptr, b, ucnt.ptr, ucnt.ptr, n + 1, st));
         FSGC_CUDA(cub::DeviceScan::ExclusiveSum(tmp.ptr, b, ucnt_big.ptr, ucnt_big.ptr, n + 1, st));
         FSGC_CUDA(units.alloc((size_t)n + (size_t)m / FSGC_SUP_SEG + 1, st));   // >= sum ceil(in/SEG)
-        FSGC_CUDA(units_big.alloc((size_t)m / FSGC_SUP_CAPW + (size_t)m / FSGC_SUP_SEG + 1, st));
+        FSGC_CUDA(units_big.alloc((size_t)n + (size_t)m / FSGC_SUP_CHUNK + 1, st));
         unit_fill<<<grid_for(n), 256, 0, st>>>(ucnt.ptr, n, units.ptr);
         FSGC_CUDA(cudaGetLastError());
         unit_fill<<<grid_for(n), 256, 0, st>>>(ucnt_big.ptr, n, units_big.ptr);
         FSGC_CUDA(cudaGetLastError());
     }
-    if (m > 0) {
+    if (m > 0 && merge_list) {
         DevBuf<uint32_t> k0, k1;
         DevBuf<int32_t> i1;
         FSGC_CUDA(k0.alloc(m, st));
         FSGC_CUDA(k1.alloc(m, st));
         FSGC_CUDA(sorder.alloc(m, st));
         FSGC_CUDA(i1.alloc(m, st));
-        support_work_keys<<<grid_for(m), 256, 0, st>>>(offs.ptr, split.ptr, osrc.ptr, odst.ptr, m, k0.ptr, sorder.ptr,
-                                                       (unsigned long long*)dnum.ptr,
-                                                       use_hash ? cap_big : (int64_t)-1);
+        support_work_keys<<<grid_for(m), 256, 0, st>>>(offs.ptr, split.ptr, osrc.ptr, odst.ptr, m, k0.ptr, sorder.ptr);
         FSGC_CUDA(cudaGetLastError());
         cub::DoubleBuffer<uint32_t> dk(k0.ptr, k1.ptr);
         cub::DoubleBuffer<int32_t> dv(sorder.ptr, i1.ptr);
@@ -506,7 +508,7 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
     // memory); FSGC_HUB_BYTES overrides), only for degree >= kHubMinDeg
     int64_t hub_base = n, hub_words = (n + 31) / 32;
     int64_t maxdeg = 0;   // the last vertex has the largest degree
-    int64_t nheavy = 0, nunits = 0, nunits_big = 0;
+    int64_t nunits = 0, nunits_big = 0, maxout_big = 0;
     DevBuf<uint32_t> hubs;
     {
         size_t free_b = 0, total_b = 0;
@@ -520,10 +522,10 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
         // first v in [n - max_hubs, n) with deg(v) >= kHubMinDeg (degrees are
         // ascending in the new ids), and the maximum degree: one synchronisation
         int64_t hv2[2] = {n, 0};
-        if (m > 0) FSGC_CUDA(cudaMemcpyAsync(&nheavy, dnum.ptr, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
-        if (m > 0 && use_hash) {   // heavy-edge count (dnum[0], from support_work_keys) and units
+        if (m > 0) {   // unit counts and the largest block-table out-degree
             FSGC_CUDA(cudaMemcpyAsync(&nunits, ucnt.ptr + n, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
             FSGC_CUDA(cudaMemcpyAsync(&nunits_big, ucnt_big.ptr + n, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
+            FSGC_CUDA(cudaMemcpyAsync(&maxout_big, dnum.ptr + 1, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
         }
         if (n > 0) {
             DevBuf<int64_t> hs;
@@ -562,12 +564,14 @@ extern "C" int fsgc_load_graph(const void* edges, int64_t E, int ib, int64_t n, 
     g->sorder = sorder.take();
     g->ssrc = ssrc.take();
     g->sdst = sdst.take();
-    g->nsup_heavy = nheavy;
+    g->nsup_merge = merge_list ? m : 0;
+    g->sup_hash = use_hash ? 1 : 0;
     g->sup_units = units.take();
     g->nsup_units = nunits;
     g->sup_units_big = units_big.take();
     g->nsup_units_big = nunits_big;
-    g->sup_cap_big = (int32_t)cap_big;
+    g->sup_capw = (int32_t)capw;
+    g->sup_maxout = maxout_big;
     g->rev = rev.take();
     g->hub_base = hub_base;
     g->hub_words = hub_words;

@@ -15,10 +15,11 @@ void fsgc_set_error(const char* fmt, ...);
         return (code);                  \
     } while (0)
 
-// support pass split (graph.cu builds the work lists, count.cu runs them)
-#define FSGC_SUP_CAPW 256        // max out(b) of a middle vertex with a small warp table
-#define FSGC_SUP_CAP 1024        // max out(b) of a middle vertex with a large warp table
-#define FSGC_SUP_SEG 128         // in-neighbours per work unit (one warp)
+// triangle listing from the middle vertex (graph.cu builds the work units,
+// count.cu runs them: support pass and triangle-core pass)
+#define FSGC_SUP_CAPW 256        // max out(b) of a middle vertex with a warp table
+#define FSGC_SUP_SEG 128         // in-neighbours per warp-table unit
+#define FSGC_SUP_CHUNK 1024      // in-neighbours per block-table unit
 
 // --------------------------------------------------------------- handles
 struct fsgc_graph {
@@ -34,28 +35,30 @@ struct fsgc_graph {
     int64_t* oofs = nullptr;     // [n+1] oriented offsets: oriented index of
                                  //       CSR position p >= split[u] is
                                  //       oofs[u] + p - split[u]
-    // support pass, wedge-hash part (count.cu support_hash_kernel): every
-    // triangle a < b < c is found from its middle vertex b.  Units = (b, k),
-    // packed b << 32 | k, ordered by b:
-    //   sup_units      1 <= out(b) <= FSGC_SUP_CAPW
-    //   sup_units_big  FSGC_SUP_CAPW < out(b) <= FSGC_SUP_CAP
-    // unit (b, k) = the k-th FSGC_SUP_SEG slice of b's in-list N-(b); one
-    // warp with its own table of N+(b) per unit
+    // Triangle listing from the MIDDLE vertex b (count.cu): every triangle
+    // a < b < c is found from b, c in N+(a) & N+(b), a in N-(b).  Units =
+    // (b, k), packed b << 32 | k, ordered by b:
+    //   sup_units      1 <= out(b) <= sup_capw: the k-th FSGC_SUP_SEG slice of
+    //                  N-(b), one warp with its own hash table of N+(b)
+    //   sup_units_big  out(b) > sup_capw: the k-th FSGC_SUP_CHUNK slice of
+    //                  N-(b), one block with a shared table of N+(b)
     uint64_t* sup_units = nullptr;   // [nsup_units]
     int64_t nsup_units = 0;
     uint64_t* sup_units_big = nullptr;   // [nsup_units_big]
     int64_t nsup_units_big = 0;
-    int32_t sup_cap_big = FSGC_SUP_CAP;   // max out(b) of a large-table middle (FSGC_SUP_CAP_BIG)
+    int32_t sup_capw = FSGC_SUP_CAPW;    // out(b) split between the two (FSGC_SUP_CAPW knob)
+    int64_t sup_maxout = 0;              // max out(b) of a block-table middle (table size)
     // rev[i - oofs[b]] = oriented index of (a, b) for the in-entry a = adj[i]
     // of row b (i in [offs[b], split[b])) -- the position of b in N+(a)
     int32_t* rev = nullptr;          // [m]
-    // support pass, merge part (support_kernel): the oriented edges (a, b)
-    // whose middle vertex b has out(b) > FSGC_SUP_CAP, sorted by merge length
-    // out(a) + out(b), with their endpoints (coalesced reads in that order)
-    int32_t* sorder = nullptr;   // [nsup_heavy]
-    int32_t* ssrc = nullptr;     // [nsup_heavy]
-    int32_t* sdst = nullptr;     // [nsup_heavy]
-    int64_t nsup_heavy = 0;
+    int32_t sup_hash = 1;            // support pass: 1 listing kernels, 0 merge kernel
+    // merge kernel (support_kernel) work list: every oriented edge (a, b)
+    // sorted by merge length out(a) + out(b), with its endpoints (only for
+    // graphs below FSGC_SUP_HASH_MIN_M edges or FSGC_SUP_MERGE_ONLY)
+    int32_t* sorder = nullptr;   // [nsup_merge]
+    int32_t* ssrc = nullptr;     // [nsup_merge]
+    int32_t* sdst = nullptr;     // [nsup_merge]
+    int64_t nsup_merge = 0;
     // hub bitmaps: vertices v >= hub_base (the highest-degree ones, ids are
     // degree ordered) have a dense n-bit adjacency bitmap (O(1) membership)
     int64_t hub_base = 0;        // == n when there are no hubs

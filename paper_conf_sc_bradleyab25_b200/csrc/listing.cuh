@@ -1,0 +1,727 @@
+// listing.cuh -- triangle listing from the MIDDLE vertex (included by
+// count.cu): the per-edge support pass and the triangle-core pass share it.
+//
+// PAPER.md Sec. 3.6 intersects the neighbour lists of the matched vertices
+// per core match; Sec. 3.3 needs, per triangle core (u, v, w), the sizes of
+// the Venn regions of e(u), e(v), e(w).  Here every triangle a < b < c
+// (degree-ordered ids, Sec. 3.1 symmetry breaking) is found from its middle
+// vertex b: c in N+(a) & N+(b) with a in N-(b) = {a < b, a ~ b} and c > b.
+// A work unit is (b, slice of N-(b)); N+(b) is staged in a shared-memory
+// hash table once per b, and for every in-neighbour a of the slice the tail
+// of N+(a) after b (b's position in N+(a) comes from graph.rev) is streamed
+// through the table.  Work: sum_a out(a)^2 / 2 probes, coalesced tail reads,
+// no per-match binary search.
+//
+//   warp tables  (out(b) <= capw = 256, the many small middles): one warp per
+//                unit with its own table; the slice's tails are concatenated
+//                (warp prefix sum) so the 32 lanes read 32 consecutive
+//                virtual elements whatever the tail lengths;
+//   block tables (out(b) > capw, the heavy middles: RMAT-26 has out(b) up to
+//                3,004): one block per unit with a table sized to the graph's
+//                largest out(b); the warps take 32 in-neighbours at a time
+//                from a block-local counter (dynamic within the block) and
+//                stream one tail at a time, kILP loads in flight per lane.
+// Units come from a global atomic queue (heavy middles first for the block
+// kernel), dealt round-robin over the shards of a multi-GPU count.
+//
+// Two visitors of the same listing (template flag TRI):
+//   support   (TRI = false): c(e) = |N(u) & N(v)| for every oriented edge:
+//             a hit (a, b, c) adds 1 to c(bc) (shared counter per table slot,
+//             flushed when the table changes), c(ac) (global reduction) and
+//             c(ab) (ballot count per in-neighbour, one add per (a, b));
+//   tri-core  (TRI = true, after the support pass): a hit is a triangle core
+//             match (u, v, w) = (a, b, c); its degrees and supports are
+//             gathered (deg / c(bc) of the N+(b) entries are staged beside
+//             the table), buffered per warp, and the buffer is flushed
+//             through the Venn diagram (Sec. 3.3) and the fringe counting
+//             function (Venn term table, else Listing 5).
+
+constexpr int kLeafCap = 64;      // leaf buffer per warp (flushed at >= 32)
+constexpr int kLeafW = 10;        // a, b, c, du, dv, dw, cuv, e(ac), cvw, pad
+constexpr int kILP = 4;           // tail loads in flight per lane (block tables)
+constexpr int kWarpTabWarps = 8;  // warps per block, warp-table kernels
+constexpr int kBlockTabWarps = 16;   // warps per block, block-table support kernel
+constexpr int kBlockTriWarps = 8;    // warps per block, block-table tri-core kernel
+
+__device__ __forceinline__ uint32_t hslot(int x, int hbits) { return ((uint32_t)x * 0x9E3779B1u) >> (32 - hbits); }
+
+// slot of x in the table, -1 if absent (open addressing, linear probing)
+__device__ __forceinline__ int hfind(const int32_t* key, int x, int hbits) {
+    const uint32_t hm = (1u << hbits) - 1;
+    uint32_t h = hslot(x, hbits);
+    int y;
+    while ((y = key[h]) != x && y != -1) h = (h + 1) & hm;
+    return y == x ? (int)h : -1;
+}
+
+// the table of N+(b): keys, kpos = position of the key in N+(b), and the
+// payload, built by `nthr` threads (a warp or a block; the caller
+// synchronises before and after).  Support: cnt[slot] = 0 (the c(b, x)
+// counters).  Tri-core: tsup[i] = c(b, x), tdeg[i] = deg(x) for the i-th
+// entry x of N+(b).
+template <bool TRI>
+__device__ __forceinline__ void table_build(const GraphDev& G, const OrientDev& O, const int* __restrict__ sup,
+                                            int b, int64_t sb, int ob, int hbits, int32_t* key, int16_t* kpos,
+                                            int32_t* cnt, int32_t* tsup, int32_t* tdeg, int tid, int nthr) {
+    const uint32_t hm = (1u << hbits) - 1;
+    const int64_t ob0 = TRI ? __ldg(O.oofs + b) : 0;
+    for (int i = tid; i < ob; i += nthr) {
+        const int x = __ldg(G.adj + sb + i);
+        uint32_t h = hslot(x, hbits);
+        while (atomicCAS(&key[h], -1, x) != -1) h = (h + 1) & hm;
+        kpos[h] = (int16_t)i;
+        if (TRI) {
+            tsup[i] = __ldg(sup + ob0 + i);
+            tdeg[i] = (int)(__ldg(G.offs + x + 1) - __ldg(G.offs + x));
+        } else {
+            cnt[h] = 0;
+        }
+    }
+}
+
+// support: add the table's c(b, x) counters to the support array
+__device__ __forceinline__ void table_flush(const OrientDev& O, int* __restrict__ sup, int b, int hbits,
+                                            const int32_t* key, const int16_t* kpos, const int32_t* cnt, int tid,
+                                            int nthr) {
+    const int64_t base = __ldg(O.oofs + b);
+    for (int h = tid; h < (1 << hbits); h += nthr)
+        if (key[h] != -1 && cnt[h]) atomicAdd(sup + base + kpos[h], cnt[h]);
+}
+
+// ------------------------------------------------------------------------
+// tri-core visitor: the per-warp leaf buffer and its flush
+struct TriCtx {
+    int q, V, nprog;
+    int proj[8];        // core position mask F (bit0 u, bit1 v, bit2 w) -> Venn bit mask
+    bool need_t;        // the anchors' Venn needs t = |N(u) & N(v) & N(w)|
+    int mindeg0, mindeg1, mindeg2;
+    int degfilter;
+    int cmask[8];       // Venn bit mask -> core position mask (bit0 u, bit1 v, bit2 w)
+};
+
+// Necessary condition for fc > 0 from the pairwise quantities alone: some
+// program whose every fringe type t' fits k_t' <= Z[A_t'] -- with
+// Z[{x}] = deg(x) - 2 and Z[{x, y}] = c(xy) - 1 exact (core vertices
+// excluded) and Z[{u, v, w}] = t <= min c(..) - 1.  Leaves that fail it have
+// fc = 0 for every program: no triple intersection, no fc evaluation.
+__device__ __forceinline__ bool tri_alive(const CoreProg& P, const TriCtx& C, int du, int dv, int dw, int cuv,
+                                          int cuw, int cvw) {
+    int z[8];
+    z[0] = 1 << 30;
+    z[1] = du - 2; z[2] = dv - 2; z[4] = dw - 2;
+    z[3] = cuv - 1; z[5] = cuw - 1; z[6] = cvw - 1;
+    z[7] = min(z[3], min(z[5], z[6]));
+    for (int pi = 0; pi < C.nprog; ++pi) {
+        const FringeProg& fp = P.prog[pi];
+        bool ok = true;
+        for (int t = 0; t < fp.s && ok; ++t) ok = (int)fp.k[t] <= z[C.cmask[fp.anch[t]]];
+        if (ok) return true;
+    }
+    return C.nprog == 0;
+}
+
+__device__ __forceinline__ void tri_ctx_init(TriCtx& C, const CoreProg& P, const WorkDesc& W) {
+    C.q = P.q;
+    C.V = 1 << P.q;
+    C.nprog = P.nprog;
+#pragma unroll
+    for (int F = 0; F < 8; ++F) {
+        int M = 0;
+        for (int b = 0; b < P.q; ++b)
+            if ((F >> P.anchor_pos[b]) & 1) M |= 1 << b;
+        C.proj[F] = M;
+    }
+#pragma unroll
+    for (int M = 0; M < 8; ++M) {
+        int cm = 0;
+        for (int b = 0; b < P.q; ++b)
+            if ((M >> b) & 1) cm |= 1 << P.anchor_pos[b];
+        C.cmask[M] = cm;
+    }
+    // Does any program's fc depend on t = |N(u) & N(v) & N(w)|?  A vertex of
+    // region F (core positions it is adjacent to) can serve the fringe types
+    // t' with A_t' inside proj[F] -- its signature.  A program's fc depends
+    // only on the sizes of its signature classes (vertices with the same
+    // signature are interchangeable), and t enters region F with sign +1
+    // (|F| odd) or -1 (|F| = 2).  So t is needed iff some program has a
+    // non-empty signature class whose signs do not cancel (e.g. a
+    // tri-fringe, or tails on all three core vertices); otherwise any t in
+    // the feasible range gives the same fc (tri_flush takes the smallest).
+    C.need_t = false;
+    for (int pi = 0; pi < P.nprog && !C.need_t; ++pi) {
+        const FringeProg& fp = P.prog[pi];
+        int sig[8], coef[8];
+        for (int F = 1; F < 8; ++F) {
+            int sg = 0;
+            for (int t = 0; t < fp.s; ++t)
+                if ((C.proj[F] & fp.anch[t]) == fp.anch[t]) sg |= 1 << t;
+            sig[F] = sg;
+            coef[F] = 0;
+        }
+        for (int F = 1; F < 8; ++F) {
+            if (!sig[F]) continue;
+            int c = 0;
+            for (int G = 1; G < 8; ++G)
+                if (sig[G] == sig[F]) c += (__popc(G) & 1) ? 1 : -1;
+            if (c != 0) C.need_t = true;
+        }
+    }
+    C.mindeg0 = P.mindeg[0];
+    C.mindeg1 = P.mindeg[1];
+    C.mindeg2 = P.mindeg[2];
+    C.degfilter = W.degfilter;
+}
+
+template <class W>
+__device__ __forceinline__ W sext(int64_t c);
+template <>
+__device__ __forceinline__ uint64_t sext<uint64_t>(int64_t c) { return (uint64_t)c; }
+template <>
+__device__ __forceinline__ u128 sext<u128>(int64_t c) { return (u128)(__int128)c; }
+
+// the Z-term table on one triangle (z[cm] = Z of the core-position set cm),
+// arithmetic mod 2^bits(W): exact when each pattern's sum over its programs
+// (a sum of products of binomials C(Z, k) bounded by the caller's bound) is
+// below 2^(bits - 9): then every row entry C(Z, j) fits with its 2-adic part
+template <class W, int NP>
+__device__ __forceinline__ void zterms_eval(const int* z, const VennDev& T, W* R, int stride, AccN<NP>& acc) {
+#pragma unroll
+    for (int cm = 1; cm < 8; ++cm) {
+        const int K = T.zmaxj[cm];
+        if (!K) continue;
+        const uint64_t n = (uint64_t)z[cm];
+        W* Rr = R + T.zbase[cm] * stride;
+        W c = 1;
+        for (int j = 1; j <= K; ++j) {
+            c = ((c * (W)(n - (uint64_t)j + 1)) >> c_tz[j]) * inv_odd(j, c);
+            Rr[(j - 1) * stride] = c;
+        }
+    }
+    W sum = 0;
+    int cur = -1;
+    for (int t = 0; t < T.zn; ++t) {
+        const ZTerm e = T.zterms[t];
+        if (e.pat != cur) {
+            if (cur >= 0) acc.add(cur, (u128)sum, false);
+            sum = 0;
+            cur = e.pat;
+        }
+        W pr = sext<W>(e.coef);
+        for (int i = 0; i < e.nf; ++i) pr *= R[e.f[i] * stride];
+        sum += pr;
+    }
+    if (cur >= 0) acc.add(cur, (u128)sum, false);
+}
+
+// Flush the warp's `cnt` buffered triangle matches (leaf[i * kLeafW + .]):
+// Venn diagram (Sec. 3.3) -- with c(xy) = |N(x) & N(y)| and
+// t = |N(u) & N(v) & N(w)| the 7 regions of e(u), e(v), e(w) (core vertices
+// excluded; each core vertex is adjacent to the other two) are
+//   uvw = t, uv = c(uv) - 1 - t, uw = c(uw) - 1 - t, vw = c(vw) - 1 - t,
+//   u = deg(u) - 2 - uv - uw - t (likewise v, w),
+// projected onto the q anchors -- then fc (Venn term table in the 64- or
+// 128-bit tier, else Listing 5 per program).  t by one triple intersection:
+// N(u), the shortest list (u has the lowest degree), scanned against N(v),
+// N(w) through hub bitmaps or galloping cursors; warp-cooperative for long
+// lists.
+template <int NP>
+__device__ __noinline__ void tri_flush(const GraphDev& G, const HubDev& H, const CoreProg& P, const VennDev& VD,
+                                       const TriCtx& C, const int* __restrict__ sup, uint32_t* leaf, int cnt,
+                                       u128* lane_rows, int lane_stride, u128* warp_rows, int lane,
+                                       AccN<NP>& acc) {
+    __syncwarp();
+    for (int base = 0; base < cnt; base += 32) {
+        const int li = base + lane;
+        const bool mine = li < cnt;
+        const uint32_t* L = leaf + li * kLeafW;
+        int lu = 0, lv = 0, lw = 0, du = 0, dv = 0, dw = 0, cuv = 0, cuw = 0, cvw = 0, t = 0;
+        if (mine) {
+            lu = (int)L[0]; lv = (int)L[1]; lw = (int)L[2];
+            du = (int)L[3]; dv = (int)L[4]; dw = (int)L[5];
+            cuv = (int)L[6]; cvw = (int)L[8];
+            cuw = __ldg(sup + L[7]);
+        }
+        // leaves whose fc is 0 for every program (necessary condition from
+        // degrees and supports) are counted as matches and skipped
+        const bool alive = mine && tri_alive(P, C, du, dv, dw, cuv, cuw, cvw);
+        // Z-term path: tier bound from the largest Z in use and the largest
+        // program (prod_t C(Z_t, k_t) <= Zmax^K); past 2^119 the leaf takes
+        // the checked Listing 5 on its Venn diagram
+        float zb = 0.f;
+        if (VD.zn && alive) {
+            const int zmax = max(max(du, dv), dw);
+            zb = (float)VD.zk * log2f((float)zmax + 1.f) + VD.slack;
+        }
+        const bool zfb = VD.zn && zb >= 119.f;
+        const bool want_t = alive && (VD.zn ? (VD.zneed7 || (zfb && C.need_t)) : C.need_t);
+        const bool heavy = want_t && du > 32;
+        if (want_t && !heavy) {
+            Cursor cv, cw;
+            cv.init(G, H, lv);
+            cw.init(G, H, lw);
+            const int64_t b0 = __ldg(G.offs + lu);
+            for (int i = 0; i < du; ++i) {
+                const int x = __ldg(G.adj + b0 + i);
+                if (cv.has(x) && cw.has(x)) ++t;
+            }
+        }
+        unsigned hb = __ballot_sync(FULLMASK, heavy);
+        while (hb) {
+            const int who = __ffs(hb) - 1;
+            hb &= hb - 1;
+            const int hu = __shfl_sync(FULLMASK, lu, who), hv = __shfl_sync(FULLMASK, lv, who);
+            const int hw = __shfl_sync(FULLMASK, lw, who), hd = __shfl_sync(FULLMASK, du, who);
+            const int64_t b0 = __ldg(G.offs + hu);
+            int tt = 0;
+            for (int s0 = 0; s0 < hd; s0 += 32) {
+                bool hit = false;
+                if (s0 + lane < hd) {
+                    const int x = __ldg(G.adj + b0 + s0 + lane);
+                    hit = member(G, H, hv, x) && member(G, H, hw, x);
+                }
+                tt += __popc(__ballot_sync(FULLMASK, hit));
+            }
+            if (lane == who) t = tt;
+        }
+        if (alive && !want_t) {   // any feasible t: the smallest keeps every region >= 0
+            t = max(max(0, cuv + cuw - du), max(cuv + cvw - dv, cuw + cvw - dw));
+        }
+        if (VD.zn) {                   // fc from the Z values (no Venn diagram)
+            const bool all64 = __all_sync(FULLMASK, !alive || zb < 55.f);
+            int z[8];
+            z[0] = 0;
+            z[1] = du - 2; z[2] = dv - 2; z[4] = dw - 2;
+            z[3] = cuv - 1; z[5] = cuw - 1; z[6] = cvw - 1;
+            z[7] = t;
+            if (alive && all64) {
+                zterms_eval<uint64_t>(z, VD, (uint64_t*)lane_rows, 2 * lane_stride, acc);
+            } else if (alive && !zfb) {
+                zterms_eval<u128>(z, VD, lane_rows, lane_stride, acc);
+            }
+            if (!__any_sync(FULLMASK, alive && zfb)) continue;
+        }
+        uint32_t vq[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+        if (alive) {
+            int R[8];
+            R[0] = 0;
+            R[7] = t;
+            R[3] = cuv - 1 - t;
+            R[5] = cuw - 1 - t;
+            R[6] = cvw - 1 - t;
+            R[1] = du - 2 - R[3] - R[5] - t;
+            R[2] = dv - 2 - R[3] - R[6] - t;
+            R[4] = dw - 2 - R[5] - R[6] - t;
+#pragma unroll
+            for (int F = 1; F < 8; ++F)
+                if (C.proj[F]) vq[C.proj[F]] += (uint32_t)R[F];
+        }
+        if (VD.zn) {                    // Z mode, fallback lanes: checked Listing 5
+            if (alive && zfb)
+                for (int pi = 0; pi < C.nprog; ++pi) {
+                    const FringeProg fp = P.prog[pi];
+                    bool o = false;
+                    const u128 f = fc_dispatch<kTriStack>(vq, C.q, fp, o);
+                    acc.add(fp.pat, f, o);
+                }
+        } else if (VD.n && VD.warp) {          // one diagram per warp, lanes over the terms
+            unsigned am = __ballot_sync(FULLMASK, alive);
+            while (am) {
+                const int l = __ffs(am) - 1;
+                am &= am - 1;
+                uint32_t vloc[8];
+#pragma unroll
+                for (int k = 0; k < 8; ++k) vloc[k] = __shfl_sync(FULLMASK, vq[k], l);
+                venn_fc_warp<kTriStack>(vloc, C.q, P, VD, warp_rows, lane, acc);
+            }
+        } else if (VD.n) {              // one diagram per lane, rows per thread
+            float bnd = 0.f;
+            if (alive) bnd = venn_bound_log2(vq, C.q, P) + VD.slack;
+            const bool all64 = __all_sync(FULLMASK, !alive || bnd < 55.f);
+            if (alive && all64) {
+                venn_terms_eval<uint64_t>(vq, C.V, VD, (uint64_t*)lane_rows, 2 * lane_stride, acc);
+            } else if (alive && bnd < 119.f) {
+                venn_terms_eval<u128>(vq, C.V, VD, lane_rows, lane_stride, acc);
+            } else if (alive) {
+                for (int pi = 0; pi < C.nprog; ++pi) {
+                    const FringeProg fp = P.prog[pi];
+                    bool o = false;
+                    const u128 f = fc_dispatch<kTriStack>(vq, C.q, fp, o);
+                    acc.add(fp.pat, f, o);
+                }
+            }
+        } else {                        // Listing 5 per program (no table)
+            if (alive)
+                for (int pi = 0; pi < C.nprog; ++pi) {
+                    const FringeProg fp = P.prog[pi];
+                    bool o = false;
+                    const u128 f = fc_dispatch<kTriStack>(vq, C.q, fp, o);
+                    acc.add(fp.pat, f, o);
+                }
+        }
+    }
+    __syncwarp();
+}
+
+// append the hits of one round (hit: this lane's candidate c is in N+(b)) to
+// the warp's leaf buffer; the caller flushes at >= 32
+__device__ __forceinline__ int tri_append(uint32_t* leaf, int cnt, bool hit, int a, int b, int c, int du, int dv,
+                                          int dw, int cuv, uint32_t eac, int cvw, int lane) {
+    const unsigned fm = __ballot_sync(FULLMASK, hit);
+    if (hit) {
+        uint32_t* L = leaf + (cnt + __popc(fm & ((1u << lane) - 1))) * kLeafW;
+        L[0] = (uint32_t)a; L[1] = (uint32_t)b; L[2] = (uint32_t)c;
+        L[3] = (uint32_t)du; L[4] = (uint32_t)dv; L[5] = (uint32_t)dw;
+        L[6] = (uint32_t)cuv; L[7] = eac; L[8] = (uint32_t)cvw;
+    }
+    return cnt + __popc(fm);
+}
+
+// ------------------------------------------------------------------------
+// warp-table kernel.  Shared memory per warp: table (key, kpos/cnt or
+// tsup/tdeg: HS = 2 * FSGC_SUP_CAPW slots), slice arrays, leaf buffer (TRI)
+template <bool TRI>
+struct WarpTabLayout {
+    static constexpr int HS = 2 * FSGC_SUP_CAPW;
+    static constexpr size_t key_b = (size_t)HS * 4;
+    static constexpr size_t kpos_b = (size_t)HS * 2;
+    static constexpr size_t pay_b = TRI ? (size_t)FSGC_SUP_CAPW * 8 : (size_t)HS * 4;   // tsup+tdeg | cnt
+    static constexpr size_t slice_b = (size_t)(FSGC_SUP_SEG + 4) * 4 + (size_t)5 * FSGC_SUP_SEG * 4;
+    static constexpr size_t leaf_b = TRI ? (size_t)kLeafCap * kLeafW * 4 : 0;
+    static constexpr size_t rows_b = TRI ? (size_t)kMaxVennRows * 16 : 0;     // warp-mode term rows
+    static constexpr size_t warp_b = key_b + kpos_b + pay_b + slice_b + leaf_b + rows_b;
+    static constexpr size_t bytes = kWarpTabWarps * warp_b;
+};
+
+template <bool TRI, int NP>
+__global__ void __launch_bounds__(kWarpTabWarps * 32) list_warp_kernel(
+    GraphDev G, OrientDev O, HubDev H, const int32_t* __restrict__ rev, const uint64_t* __restrict__ units,
+    int64_t nunits, int* __restrict__ sup, unsigned long long* queue, int shard, int nshards, const __grid_constant__ CoreProg P,
+    WorkDesc W, const __grid_constant__ VennDev VD, const Sink S) {
+    typedef WarpTabLayout<TRI> Lay;
+    extern __shared__ __align__(16) unsigned char s_lw[];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    unsigned char* tb = s_lw + (size_t)w * Lay::warp_b;
+    int32_t* key = reinterpret_cast<int32_t*>(tb);
+    int16_t* kpos = reinterpret_cast<int16_t*>(tb + Lay::key_b);
+    int32_t* pay0 = reinterpret_cast<int32_t*>(tb + Lay::key_b + Lay::kpos_b);   // cnt[slot] | tsup[pos]
+    int32_t* pay1 = pay0 + FSGC_SUP_CAPW;                                         // - | tdeg[pos]
+    unsigned char* wb = tb + Lay::key_b + Lay::kpos_b + Lay::pay_b;
+    int32_t* pre = reinterpret_cast<int32_t*>(wb);                           // [SEG + 4]
+    uint32_t* q0 = reinterpret_cast<uint32_t*>(wb + (FSGC_SUP_SEG + 4) * 4);  // tail start per in-entry
+    uint32_t* da = q0 + FSGC_SUP_SEG;                                        // split[a] - oofs[a]
+    int32_t* ea = reinterpret_cast<int32_t*>(da + FSGC_SUP_SEG);             // e(ab) | a
+    int32_t* xa = ea + FSGC_SUP_SEG;                                         // c(ab) count | deg a
+    int32_t* ya = xa + FSGC_SUP_SEG;                                         // - | c(ab)
+    uint32_t* leaf = reinterpret_cast<uint32_t*>(wb + Lay::slice_b);
+    u128* wrows = reinterpret_cast<u128*>(wb + Lay::slice_b + Lay::leaf_b);
+    u128* lrows = reinterpret_cast<u128*>(s_lw + Lay::bytes) + threadIdx.x;  // lane-mode term rows
+
+    AccN<NP> acc;
+    acc.init();
+    unsigned long long nmatch = 0;
+    TriCtx C;
+    if (TRI) tri_ctx_init(C, P, W);
+    int cnt = 0;
+    int prev_b = -1, ob = 0, hbits = 5, degb = 0;
+    int64_t sb = 0;
+    const int64_t mine = nunits > shard ? (nunits - shard + nshards - 1) / nshards : 0;
+    for (;;) {
+        unsigned long long jq = 0;
+        if (lane == 0) jq = atomicAdd(queue, 1ull);
+        jq = __shfl_sync(FULLMASK, jq, 0);
+        if ((int64_t)jq >= mine) break;
+        const int64_t tu = (int64_t)jq * nshards + shard;
+        const uint64_t un = __ldg(units + tu);
+        const int b = (int)(un >> 32), k = (int)(un & 0xffffffffu);
+        if (b != prev_b) {                    // (re)build the table of N+(b)
+            if (!TRI && prev_b >= 0) {
+                __syncwarp();
+                table_flush(O, sup, prev_b, hbits, key, kpos, pay0, lane, 32);
+            }
+            const int64_t ob_ = __ldg(G.offs + b);
+            sb = __ldg(O.split + b);
+            ob = (int)(__ldg(G.offs + b + 1) - sb);
+            degb = (int)(__ldg(G.offs + b + 1) - ob_);
+            hbits = 5;
+            while ((1 << hbits) < 2 * ob) ++hbits;
+            __syncwarp();
+            for (int i = lane; i < (1 << hbits); i += 32) key[i] = -1;
+            __syncwarp();
+            table_build<TRI>(G, O, sup, b, sb, ob, hbits, key, kpos, pay0, pay0, pay1, lane, 32);
+            prev_b = b;
+            __syncwarp();
+        }
+        if (TRI && W.degfilter && degb < C.mindeg1) continue;
+        const int64_t ib0 = __ldg(G.offs + b) + (int64_t)k * FSGC_SUP_SEG;
+        const int len = (int)min((int64_t)FSGC_SUP_SEG, sb - ib0);
+        const int64_t rbase = ib0 - __ldg(O.oofs + b);
+        // slice setup: per in-entry a the start q0 of its tail (after b in
+        // N+(a)) and the tail length; exclusive scan of the lengths -> pre
+        int carry = 0;
+        for (int j0 = 0; j0 < len; j0 += 32) {
+            const int j = j0 + lane;
+            int Lt = 0;
+            if (j < len) {
+                const int a = __ldg(G.adj + ib0 + j);
+                const int e = __ldg(rev + rbase + j);
+                const int64_t sa = __ldg(O.split + a), oa = __ldg(O.oofs + a);
+                const int64_t q = sa + (e - oa) + 1;
+                Lt = (int)(__ldg(G.offs + a + 1) - q);
+                q0[j] = (uint32_t)q;
+                da[j] = (uint32_t)(sa - oa);
+                if (TRI) {
+                    const int dga = (int)(__ldg(G.offs + a + 1) - __ldg(G.offs + a));
+                    ea[j] = a;
+                    xa[j] = dga;
+                    ya[j] = __ldg(sup + e);
+                    if (W.degfilter && dga < C.mindeg0) Lt = 0;
+                    if (ya[j] == 0) Lt = 0;          // no triangle on (a, b)
+                } else {
+                    ea[j] = e;
+                    xa[j] = 0;
+                }
+            }
+            int x = Lt;                       // inclusive warp scan
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const int y = __shfl_up_sync(FULLMASK, x, o);
+                if (lane >= o) x += y;
+            }
+            if (j < len) pre[j] = carry + x - Lt;
+            carry += __shfl_sync(FULLMASK, x, 31);
+        }
+        if (lane == 0) pre[len] = carry;
+        __syncwarp();
+        const int total = carry;
+        int lo = 0;                           // monotone: last j with pre[j] <= idx
+        for (int v0 = 0; v0 < total; v0 += 64) {
+            int jj[2], cc[2];
+            uint32_t pp[2];
+            bool ok[2];
+#pragma unroll
+            for (int r = 0; r < 2; ++r) {
+                const int idx = v0 + 32 * r + lane;
+                ok[r] = idx < total;
+                jj[r] = 0; pp[r] = 0; cc[r] = -1;
+                if (ok[r]) {
+                    int l2 = lo, hi = len;
+                    while (hi - l2 > 1) {
+                        const int mid = (l2 + hi) >> 1;
+                        if (pre[mid] <= idx) l2 = mid; else hi = mid;
+                    }
+                    lo = l2;
+                    jj[r] = l2;
+                    pp[r] = q0[l2] + (uint32_t)(idx - pre[l2]);
+                    cc[r] = __ldg(G.adj + pp[r]);
+                }
+            }
+#pragma unroll
+            for (int r = 0; r < 2; ++r) {
+                const int h = ok[r] ? hfind(key, cc[r], hbits) : -1;
+                bool hit = h >= 0;
+                if (TRI) {
+                    int dw = 0, cvw = 0;
+                    if (hit) {
+                        const int kk = kpos[h];
+                        dw = pay1[kk];
+                        cvw = pay0[kk];
+                        if (W.degfilter && dw < C.mindeg2) hit = false;
+                    }
+                    cnt = tri_append(leaf, cnt, hit, ea[jj[r]], b, cc[r], xa[jj[r]], degb, dw, ya[jj[r]],
+                                     pp[r] - da[jj[r]], cvw, lane);
+                    if (cnt >= 32) {
+                        tri_flush<NP>(G, H, P, VD, C, sup, leaf, cnt, lrows, blockDim.x, wrows, lane, acc);
+                        if (lane == 0) nmatch += cnt;
+                        cnt = 0;
+                    }
+                } else {
+                    const unsigned hmask = __ballot_sync(FULLMASK, hit);
+                    if (hit) {
+                        atomicAdd(&pay0[h], 1);                              // c(bc)
+                        atomicAdd(sup + (pp[r] - da[jj[r]]), 1);             // c(ac)
+                        const unsigned peers = __match_any_sync(hmask, jj[r]);   // c(ab): one add per a
+                        if ((peers & ((1u << lane) - 1)) == 0) atomicAdd(&xa[jj[r]], __popc(peers));
+                    }
+                }
+            }
+        }
+        __syncwarp();
+        if (!TRI) {
+            for (int j = lane; j < len; j += 32)
+                if (xa[j]) atomicAdd(sup + ea[j], xa[j]);
+        }
+        __syncwarp();
+    }
+    if (TRI) {
+        if (cnt) {
+            tri_flush<NP>(G, H, P, VD, C, sup, leaf, cnt, lrows, blockDim.x, wrows, lane, acc);
+            if (lane == 0) nmatch += cnt;
+        }
+        block_publish<NP>(acc, nmatch, S);
+    } else if (prev_b >= 0) {
+        __syncwarp();
+        table_flush(O, sup, prev_b, hbits, key, kpos, pay0, lane, 32);
+    }
+}
+
+// ------------------------------------------------------------------------
+// block-table kernel: the heavy middles.  Shared memory: the table of N+(b)
+// (HS = pow2 >= 2 * max out(b) slots: key + payload), the block's unit and
+// in-neighbour counters, per warp a leaf buffer and term rows (TRI).
+// table bytes for hbits_max / max out(b): key + kpos per slot, then the
+// payload (support: cnt per slot; tri-core: tsup + tdeg per position)
+__host__ __device__ inline size_t blocktab_table_bytes(int hs, int maxout, bool tri) {
+    const size_t b = (size_t)hs * 6 + (tri ? (size_t)maxout * 8 : (size_t)hs * 4);
+    return (b + 15) & ~(size_t)15;
+}
+__host__ __device__ inline size_t blocktab_warp_bytes(bool tri) {
+    return tri ? (size_t)kLeafCap * kLeafW * 4 + (size_t)kMaxVennRows * 16 : 0;
+}
+
+template <bool TRI, int NP>
+__global__ void __launch_bounds__((TRI ? kBlockTriWarps : kBlockTabWarps) * 32) list_block_kernel(
+    GraphDev G, OrientDev O, HubDev H, const int32_t* __restrict__ rev, const uint64_t* __restrict__ units,
+    int64_t nunits, int hbits_max, int maxout, int* __restrict__ sup, unsigned long long* queue, int shard, int nshards,
+    const __grid_constant__ CoreProg P, WorkDesc W, const __grid_constant__ VennDev VD, const Sink S) {
+    constexpr int NWB = TRI ? kBlockTriWarps : kBlockTabWarps;
+    extern __shared__ __align__(16) unsigned char s_lb[];
+    __shared__ long long s_unit;
+    __shared__ int s_next;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, tid = threadIdx.x, nthr = blockDim.x;
+    const int HS = 1 << hbits_max;
+    const size_t tab_b = blocktab_table_bytes(HS, maxout, TRI);
+    int32_t* key = reinterpret_cast<int32_t*>(s_lb);
+    int16_t* kpos = reinterpret_cast<int16_t*>(key + HS);
+    int32_t* pay0 = reinterpret_cast<int32_t*>(kpos + HS);   // cnt[slot] | tsup[pos]
+    int32_t* pay1 = pay0 + maxout;                            // - | tdeg[pos]
+    unsigned char* wb = s_lb + tab_b + (size_t)w * blocktab_warp_bytes(TRI);
+    uint32_t* leaf = reinterpret_cast<uint32_t*>(wb);
+    u128* wrows = reinterpret_cast<u128*>(wb + (size_t)kLeafCap * kLeafW * 4);
+    u128* lrows = reinterpret_cast<u128*>(s_lb + tab_b + NWB * blocktab_warp_bytes(TRI)) + tid;
+
+    AccN<NP> acc;
+    acc.init();
+    unsigned long long nmatch = 0;
+    TriCtx C;
+    if (TRI) tri_ctx_init(C, P, W);
+    int cnt = 0;
+    int cur_b = -1, ob = 0, hbits = 5, degb = 0;
+    int64_t sb = 0;
+    const int64_t mine = nunits > shard ? (nunits - shard + nshards - 1) / nshards : 0;
+    for (;;) {
+        if (tid == 0) {
+            const long long jq = (long long)atomicAdd(queue, 1ull);
+            s_unit = jq < mine ? (long long)__ldg(units + (nunits - 1 - (jq * nshards + shard))) : -1ll;
+            s_next = 0;
+        }
+        __syncthreads();
+        const long long un = s_unit;
+        if (un < 0) break;
+        const int b = (int)((unsigned long long)un >> 32), k = (int)(un & 0xffffffffll);
+        if (b != cur_b) {                      // (re)build the block's table of N+(b)
+            if (!TRI && cur_b >= 0) table_flush(O, sup, cur_b, hbits, key, kpos, pay0, tid, nthr);
+            const int64_t ob_ = __ldg(G.offs + b);
+            sb = __ldg(O.split + b);
+            ob = (int)(__ldg(G.offs + b + 1) - sb);
+            degb = (int)(__ldg(G.offs + b + 1) - ob_);
+            hbits = 5;
+            while ((1 << hbits) < 2 * ob) ++hbits;
+            __syncthreads();
+            for (int i = tid; i < (1 << hbits); i += nthr) key[i] = -1;
+            __syncthreads();
+            table_build<TRI>(G, O, sup, b, sb, ob, hbits, key, kpos, pay0, pay0, pay1, tid, nthr);
+            cur_b = b;
+            __syncthreads();
+        }
+        const bool skip = TRI && W.degfilter && degb < C.mindeg1;
+        const int64_t ib0 = __ldg(G.offs + b) + (int64_t)k * FSGC_SUP_CHUNK;
+        const int len = skip ? 0 : (int)min((int64_t)FSGC_SUP_CHUNK, sb - ib0);
+        const int64_t rbase = ib0 - __ldg(O.oofs + b);
+        for (;;) {
+            int j0 = 0;
+            if (lane == 0) j0 = atomicAdd(&s_next, 32);
+            j0 = __shfl_sync(FULLMASK, j0, 0);
+            if (j0 >= len) break;
+            const int j = j0 + lane;
+            int64_t qa = 0, dA = 0;
+            int La = 0, e = 0, a = 0, dga = 0, cab = 0;
+            if (j < len) {
+                a = __ldg(G.adj + ib0 + j);
+                e = __ldg(rev + rbase + j);
+                const int64_t sa = __ldg(O.split + a), oa = __ldg(O.oofs + a);
+                qa = sa + (e - oa) + 1;
+                La = (int)(__ldg(G.offs + a + 1) - qa);
+                dA = sa - oa;
+                if (TRI) {
+                    dga = (int)(__ldg(G.offs + a + 1) - __ldg(G.offs + a));
+                    cab = __ldg(sup + e);
+                    if ((W.degfilter && dga < C.mindeg0) || cab == 0) La = 0;
+                }
+            }
+            const int nj = min(32, len - j0);
+            for (int tt = 0; tt < nj; ++tt) {
+                const int Lt = __shfl_sync(FULLMASK, La, tt);
+                if (Lt == 0) continue;
+                const int64_t qt = __shfl_sync(FULLMASK, qa, tt);
+                const int64_t dt = __shfl_sync(FULLMASK, dA, tt);
+                int at = 0, dat = 0, cabt = 0;
+                if (TRI) {
+                    at = __shfl_sync(FULLMASK, a, tt);
+                    dat = __shfl_sync(FULLMASK, dga, tt);
+                    cabt = __shfl_sync(FULLMASK, cab, tt);
+                }
+                int hits = 0;
+                for (int o0 = 0; o0 < Lt; o0 += 32 * kILP) {
+                    int cc[kILP];
+#pragma unroll
+                    for (int r = 0; r < kILP; ++r) {
+                        const int o = o0 + 32 * r + lane;
+                        cc[r] = o < Lt ? __ldg(G.adj + qt + o) : -1;
+                    }
+#pragma unroll
+                    for (int r = 0; r < kILP; ++r) {
+                        const int h = cc[r] >= 0 ? hfind(key, cc[r], hbits) : -1;
+                        bool hit = h >= 0;
+                        const int64_t pos = qt + o0 + 32 * r + lane;
+                        if (TRI) {
+                            int dw = 0, cvw = 0;
+                            if (hit) {
+                                const int kk = kpos[h];
+                                dw = pay1[kk];
+                                cvw = pay0[kk];
+                                if (W.degfilter && dw < C.mindeg2) hit = false;
+                            }
+                            cnt = tri_append(leaf, cnt, hit, at, b, cc[r], dat, degb, dw, cabt,
+                                             (uint32_t)(pos - dt), cvw, lane);
+                            if (cnt >= 32) {
+                                tri_flush<NP>(G, H, P, VD, C, sup, leaf, cnt, lrows, nthr, wrows, lane, acc);
+                                if (lane == 0) nmatch += cnt;
+                                cnt = 0;
+                            }
+                        } else {
+                            if (hit) {
+                                atomicAdd(&pay0[h], 1);                  // c(bc)
+                                atomicAdd(sup + (pos - dt), 1);          // c(ac)
+                            }
+                            hits += __popc(__ballot_sync(FULLMASK, hit));
+                        }
+                    }
+                }
+                if (!TRI) {
+                    const int et = __shfl_sync(FULLMASK, e, tt);
+                    if (lane == 0 && hits) atomicAdd(sup + et, hits);   // c(ab)
+                }
+            }
+        }
+        __syncthreads();
+    }
+    if (TRI) {
+        if (cnt) {
+            tri_flush<NP>(G, H, P, VD, C, sup, leaf, cnt, lrows, nthr, wrows, lane, acc);
+            if (lane == 0) nmatch += cnt;
+        }
+        block_publish<NP>(acc, nmatch, S);
+    } else if (cur_b >= 0) {
+        table_flush(O, sup, cur_b, hbits, key, kpos, pay0, tid, nthr);
+    }
+}

@@ -26,12 +26,16 @@ METRICS = [
     "sm__warps_active.avg.pct_of_peak_sustained_active", "launch__registers_per_thread",
     "launch__grid_size", "launch__block_size", "smsp__inst_executed.sum",
     "smsp__thread_inst_executed_per_inst_executed.ratio", "sm__cycles_active.avg",
-    "sm__cycles_active.max", "gpc__cycles_elapsed.max",
+    "sm__cycles_active.max", "gpc__cycles_elapsed.max", "smsp__issue_active.avg.pct_of_peak_sustained_active",
+    "lts__t_sector_hit_rate.pct", "smsp__warps_eligible.avg.per_cycle_active",
 ]
 
 
 def short(name):
     import re
+    m = re.search(r"(list_(?:warp|block)_kernel)<(true|false|1|0)", name)
+    if m:
+        return f"{m.group(1)}<{'tri' if m.group(2) in ('true', '1') else 'support'}>"
     m = re.search(r"support_hash_kernel<\d+>", name)
     if m:
         return m.group(0)

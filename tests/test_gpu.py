@@ -41,12 +41,18 @@ _cache = {}
 # the support pass's two algorithms: the merge kernel (graphs below 2^20
 # edges by default) and the wedge-hash kernels (every larger graph: configs[2],
 # [3], [4]) -- FSGC_SUP_HASH_MIN_M is read at every fsgc_load_graph
-SUP_MODES = {"merge": str(1 << 40), "wedge-hash": "0"}
+# "block-tables": the listing kernels with the warp-table cap lowered to 4, so
+# every middle vertex with out(b) > 4 takes the block-table kernels (on the
+# bench graphs those are the heavy middles, out(b) up to 3,004 at RMAT-26)
+SUP_MODES = {"merge": {"FSGC_SUP_HASH_MIN_M": str(1 << 40)},
+             "wedge-hash": {"FSGC_SUP_HASH_MIN_M": "0"},
+             "block-tables": {"FSGC_SUP_HASH_MIN_M": "0", "FSGC_SUP_CAPW": "4"}}
 
 
 @pytest.fixture(params=sorted(SUP_MODES))
 def sup_mode(request, monkeypatch):
-    monkeypatch.setenv("FSGC_SUP_HASH_MIN_M", SUP_MODES[request.param])
+    for k, v in SUP_MODES[request.param].items():
+        monkeypatch.setenv(k, v)
     return request.param
 
 
@@ -336,7 +342,7 @@ def test_edge_core_counts_beyond_64_bits():
         assert not r.overflow and r.count == oracle.fringe_count(gadj, P.n, P.edges, P.core), P.name
 
 
-@pytest.mark.parametrize("algo", ["merge", "wedge-hash"])
+@pytest.mark.parametrize("algo", ["merge", "wedge-hash", "block-tables"])
 def test_sharded_support_stages_sum_to_whole(algo, monkeypatch):
     """FSGC_FLAG_SHARD_SUPPORT: each shard lists its interleaved part of the
     triangles into a partial support array; the SUM of the partial arrays
@@ -345,7 +351,8 @@ def test_sharded_support_stages_sum_to_whole(algo, monkeypatch):
     an edge-core, a triangle-core and a general-core pass in one plan, with
     either support algorithm (the hash kernels deal their units)."""
     from paper_conf_sc_bradleyab25_b200 import _lib
-    monkeypatch.setenv("FSGC_SUP_HASH_MIN_M", "0" if algo == "wedge-hash" else str(1 << 40))
+    for k, v in SUP_MODES[algo].items():
+        monkeypatch.setenv(k, v)
     n, e, _ = workload("pl2k")
     g = F.fsgc_load_graph(e, n)
     pats = [F.compile_named(PATTERNS[x]) for x in ["2-tailed-triangle", "tricore+3f", "k4core+2f", "cycle4"]]
@@ -482,15 +489,19 @@ def test_wedge_hash_support_equals_merge(wl, monkeypatch):
     names = ["2-tailed-triangle", "tricore+3f", "k4core+2f"]
     pats = [F.compile_named(PATTERNS[x]) for x in names]
     out = []
-    for thr in ("0", str(1 << 40)):
-        monkeypatch.setenv("FSGC_SUP_HASH_MIN_M", thr)
+    for mode in ("wedge-hash", "block-tables", "merge"):
+        for k in ("FSGC_SUP_HASH_MIN_M", "FSGC_SUP_CAPW"):
+            monkeypatch.delenv(k, raising=False)
+        for k, v in SUP_MODES[mode].items():
+            monkeypatch.setenv(k, v)
         g = F.fsgc_load_graph(e, n)
         plan = F.Plan(g, pats)
         plan.enqueue()
         torch.cuda.synchronize()
         out.append((plan.support().clone(), [r.raw for r in plan.decode()]))
-    assert torch.equal(out[0][0], out[1][0])
-    assert out[0][1] == out[1][1]
+    for o in out[1:]:
+        assert torch.equal(out[0][0], o[0])
+        assert out[0][1] == o[1]
 
 
 def _one_count_subprocess(wl, names, env_extra):
@@ -549,7 +560,9 @@ def _c_count(scale, P):
 
 
 RMAT_CASES = [
-    (12, ["triangle", "1-tailed-triangle", "3-tailed-triangle", "tricore+1f", "tricore+3f", "tricore+6f"]),
+    (12, ["triangle", "1-tailed-triangle", "3-tailed-triangle", "tricore+1f", "tricore+3f", "tricore+6f",
+          "triangle/tricore", "tricore+2f", "2-tailed-triangle/tricore", "4-tailed-triangle/tricore",
+          "diamond/tricore"]),
     (8, ["fig4"]),
     (9, ["clique4", "k4core+2f", "diamondcore+3f", "cycle4", "c4core+2f", "diamond"]),
 ]
@@ -565,3 +578,36 @@ def test_rmat_hubs_symmetry_broken_vs_c_oracle(case, sup_mode):
     for P, r in zip(pats, res):
         want = _c_count(scale, P)
         assert not r.overflow and r.count == want, (scale, P.name, r.count, want)
+
+
+def _bench_line(args, nproc=None, extra_env=None):
+    import json
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, **(extra_env or {}))
+    if nproc:
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={nproc}",
+               "--master-addr=127.0.0.1", f"--master-port={29600 + random.Random().randint(0, 2000)}",
+               os.path.join(root, "bench.py")] + args
+    else:
+        cmd = [sys.executable, os.path.join(root, "bench.py")] + args
+    out = subprocess.run(cmd, env=env, capture_output=True, text=True, timeout=900, cwd=root)
+    assert out.returncode == 0, out.stderr[-3000:]
+    lines = [ln for ln in out.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, out.stdout[-2000:]
+    return json.loads(lines[0])
+
+
+@pytest.mark.parametrize("wl", ["pl2k", "internet"])
+def test_bench_torchrun_two_ranks_equals_one(wl):
+    """bench.py under torchrun with 2 ranks (FSGC_BENCH_BACKEND=gloo: both
+    ranks share this box's GPU; the product path is NCCL) reports the same
+    counts as the single-process run, and the N=2 line is well formed."""
+    args = ["--workload", wl, "--steps", "3", "--warmup", "3", "--no-e2e", "--no-cpu-baseline",
+            "--no-per-config"]
+    one = _bench_line(args + ["--gpus", "1"])
+    two = _bench_line(args + ["--gpus", "2"], nproc=2, extra_env={"FSGC_BENCH_BACKEND": "gloo"})
+    assert one["config"]["counts"] == two["config"]["counts"]
+    assert two["n_gpus"] == 2 and one["n_gpus"] == 1
+    assert two["config"]["core_matches_per_step"] == one["config"]["core_matches_per_step"]
