@@ -394,6 +394,7 @@ def per_config_block(F, dev, flush, skip):
                                "overflow": r.overflow, "count_time_s": pms / 1e3,
                                "core_matches": pr[0].core_matches,
                                "core_matches_per_s": pr[0].core_matches / (pms / 1e3)}
+            log(f"per-config {wl}: batched {ms:.2f} ms")
             out.append({"workload": WORKLOAD_DESC[wl], "graph": {"n": n, "m": g.m, "max_degree": g.max_degree},
                         "batched": {"count_time_s": ms / 1e3, "core_matches": cm,
                                     "core_matches_per_s": cm / (ms / 1e3), "edges_per_s": g.m / (ms / 1e3),
@@ -405,6 +406,14 @@ def per_config_block(F, dev, flush, skip):
         except Exception as ex:  # a failing side config must not hide the headline line
             out.append({"workload": wl, "error": repr(ex)[:300]})
     return out
+
+
+T0 = time.perf_counter()
+
+
+def log(msg):
+    """progress on stderr (the JSON line stays the only stdout output)"""
+    print(f"[bench {time.perf_counter() - T0:8.1f}s] {msg}", file=sys.stderr, flush=True)
 
 
 def main():
@@ -440,10 +449,13 @@ def main():
         e_dev = e.contiguous()
         e_host = e_dev.cpu().pin_memory()
     del e
+    log(f"workload {args.workload}: n={n} edges={e_dev.shape[0]}")
     st_graph = listing_stats(n, e_dev)
     g = F.fsgc_load_graph(e_dev, n)
+    log(f"graph loaded: m={g.m} max_degree={g.max_degree}")
     cps = [F.compile_named(P) for P in pats]
     core_matches, _ = pass_core_matches(F, g, cps)
+    log(f"core matches per step: {core_matches}")
 
     stream = torch.cuda.current_stream()
     if world > 1:
@@ -474,6 +486,7 @@ def main():
     flush = torch.empty(64 * 1024 * 1024, dtype=torch.int32, device=dev)   # 256 MiB > 126 MB L2
     for _ in range(args.warmup):
         res = step()
+        log("warm-up step done")
     counts = [r.count for r in res]
     ref = F.fsgc_count_distributed(g, cps) if world > 1 else F.fsgc_count(g, cps)   # the synchronous API agrees
     assert [r.count for r in ref] == counts, (counts, [r.count for r in ref])
@@ -504,6 +517,7 @@ def main():
             ev1[s].record(stream)
             torch.cuda.synchronize()
         assert [r.count for r in res] == counts
+        log(f"timed step {s}: {ev0[s].elapsed_time(ev1[s]):.1f} ms")
         passes = {}
         for r in res:
             passes[r.pass_index] = r
@@ -589,6 +603,7 @@ def main():
             torch.cuda.synchronize()
             assert [x.count for x in r2] == counts
             g2.free()
+            log(f"e2e step {s}: {a.elapsed_time(b):.1f} ms")
             if s >= 1:
                 tms.append(a.elapsed_time(b))
         et = sum(tms)
@@ -604,6 +619,7 @@ def main():
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         csr = host_csr(n, e_dev)
         maps, secs, nr, threads = oracle_cpu_sample(csr, pats, args.cpu_budget)
+        log(f"cpu baseline: {nr} roots in {secs:.1f} s")
         del csr
         cpu = {"value": maps / secs, "unit": UNIT, "cores": threads, "kind": "oracle",
                "sample": f"{nr} seeded random root vertices (degree <= 20000) x {len(pats)} patterns "
