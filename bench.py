@@ -229,7 +229,7 @@ def oracle_cpu_sample(csr, pats, budget_s, seed=0, max_deg=20000, nroots=None):
         cedges = [(rel[x], rel[y]) for x, y in P.edges if x in rel and y in rel]
         decs.append((P, cs[0], oracle.automorphism_count(len(cs), cedges)))
     matches, done, t0 = 0.0, 0, time.perf_counter()
-    batch = 256
+    batch = 4   # doubled per batch: the budget check stays fine-grained on hub-heavy graphs
     while done < len(roots):
         chunk = roots[done:done + batch]
         for P, pv, autc in decs:

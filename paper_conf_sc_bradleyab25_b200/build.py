@@ -20,8 +20,11 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-O3", "-I", CSRC]
 
-SOURCES = ["pattern.cpp", "graph.cu", "count.cu"]
-HEADERS = ["internal.h", "devbuf.cuh", "u128.cuh", "fc.cuh", "listing.cuh"]
+# (source, object, extra flags): the counting kernels build once per
+# accumulator class NP (count_np.cu -DFSGC_NPV=NP), all objects in parallel
+SOURCES = [("pattern.cpp", "pattern.cpp.o", []), ("graph.cu", "graph.cu.o", []), ("count.cu", "count.cu.o", [])] + \
+          [("count_np.cu", f"count_np{v}.cu.o", [f"-DFSGC_NPV={v}"]) for v in (1, 2, 4, 8, 16)]
+HEADERS = ["internal.h", "devbuf.cuh", "u128.cuh", "fc.cuh", "listing.cuh", "count_dev.cuh"]
 
 
 def _newer(src, dst):
@@ -32,22 +35,31 @@ def build(force=False, verbose=False):
     os.makedirs(OUT, exist_ok=True)
     hdr_paths = [os.path.join(CSRC, h) for h in HEADERS]
     hdr_paths.append(os.path.join(os.path.dirname(PKG), "include", "fsgc.h"))
-    objs = []
-    for s in SOURCES:
+    objs, cmds = [], []
+    for s, o, extra in SOURCES:
         src = os.path.join(CSRC, s)
-        obj = os.path.join(OUT, s + ".o")
+        obj = os.path.join(OUT, o)
         objs.append(obj)
         stale = force or _newer(src, obj) or any(_newer(h, obj) for h in hdr_paths)
         if not stale:
             continue
-        cmd = [NVCC] + ARCH + COMMON + ["-c", src, "-o", obj]
         if s.endswith(".cu"):
-            cmd += ["-Xptxas", "-v"] if verbose else []
+            cmd = [NVCC] + ARCH + COMMON + extra + ["-c", src, "-o", obj] + (["-Xptxas", "-v"] if verbose else [])
         else:
-            cmd = [NVCC, "-x", "cu"] + ARCH + COMMON + ["-c", src, "-o", obj]
+            cmd = [NVCC, "-x", "cu"] + ARCH + COMMON + extra + ["-c", src, "-o", obj]
+        cmds.append(cmd)
+    from concurrent.futures import ThreadPoolExecutor
+
+    def run(cmd):
         if verbose:
             print(" ".join(cmd), flush=True)
-        subprocess.run(cmd, check=True)
+        return subprocess.run(cmd, capture_output=not verbose, text=True)
+
+    with ThreadPoolExecutor(max_workers=max(1, min(len(cmds), os.cpu_count() or 1))) as ex:
+        for cmd, r in zip(cmds, ex.map(run, cmds)):
+            if r.returncode != 0:
+                sys.stderr.write((r.stderr or "") + (r.stdout or ""))
+                raise subprocess.CalledProcessError(r.returncode, cmd)
     if force or any(_newer(o, LIB) for o in objs):
         cmd = [NVCC] + ARCH + ["-shared", "-cudart", "static", "-Xcompiler", "-fPIC", "-o", LIB] + objs
         if verbose:

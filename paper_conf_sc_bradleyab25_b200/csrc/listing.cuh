@@ -37,7 +37,7 @@
 //             function (Venn term table, else Listing 5).
 
 constexpr int kLeafCap = 64;      // leaf buffer per warp (flushed at >= 32)
-constexpr int kLeafW = 10;        // a, b, c, du, dv, dw, cuv, e(ac), cvw, pad
+constexpr int kLeafW = 10;        // a, b, c, du, dv, dw, cuv, cuw, cvw, pad
 constexpr int kILP = 4;           // tail loads in flight per lane (block tables)
 constexpr int kWarpTabWarps = 8;  // warps per block, warp-table kernels
 constexpr int kBlockTabWarps = 16;   // warps per block, block-table support kernel
@@ -179,38 +179,56 @@ __device__ __forceinline__ uint64_t sext<uint64_t>(int64_t c) { return (uint64_t
 template <>
 __device__ __forceinline__ u128 sext<u128>(int64_t c) { return (u128)(__int128)c; }
 
+// Z[cm] of one triangle leaf by core-position mask (registers, no dynamic
+// indexing: a select chain)
+__device__ __forceinline__ uint64_t zsel(const int (&z)[8], int cm) {
+    int r = z[1];
+#pragma unroll
+    for (int k = 2; k < 8; ++k) r = cm == k ? z[k] : r;
+    return (uint64_t)r;
+}
+
+// C(n, j) mod 2^bits(W) by the exact-division chain C(n, i) = C(n, i-1) (n-i+1) / i
+// (division by the odd part of i via its inverse, by the 2-power by a shift);
+// exact when C(n, i) * i fits for every i <= j -- the tier bound of the caller
+template <class W>
+__device__ __forceinline__ W binom_fly(uint64_t n, int j) {
+    W c = (W)n;
+    for (int i = 2; i <= j; ++i) c = ((c * (W)(n - (uint64_t)i + 1)) >> c_tz[i]) * inv_odd(i, c);
+    return c;
+}
+
 // the Z-term table on one triangle (z[cm] = Z of the core-position set cm),
 // arithmetic mod 2^bits(W): exact when each pattern's sum over its programs
 // (a sum of products of binomials C(Z, k) bounded by the caller's bound) is
-// below 2^(bits - 9): then every row entry C(Z, j) fits with its 2-adic part
+// below 2^(bits - 9): then every binomial C(Z, j) fits with its 2-adic part.
+// Terms are grouped by pattern, so the accumulator index is static (the
+// pattern loop is unrolled) and no binomial rows are kept: each factor is
+// evaluated where it is used.
 template <class W, int NP>
-__device__ __forceinline__ void zterms_eval(const int* z, const VennDev& T, W* R, int stride, AccN<NP>& acc) {
+__device__ __forceinline__ void zterms_eval(const int (&z)[8], const VennDev& T, AccN<NP>& acc) {
 #pragma unroll
-    for (int cm = 1; cm < 8; ++cm) {
-        const int K = T.zmaxj[cm];
-        if (!K) continue;
-        const uint64_t n = (uint64_t)z[cm];
-        W* Rr = R + T.zbase[cm] * stride;
-        W c = 1;
-        for (int j = 1; j <= K; ++j) {
-            c = ((c * (W)(n - (uint64_t)j + 1)) >> c_tz[j]) * inv_odd(j, c);
-            Rr[(j - 1) * stride] = c;
+    for (int p = 0; p < NP; ++p) {
+        const int t0 = T.zoff[p], t1 = T.zoff[p + 1];
+        if (t0 == t1) continue;
+        W sum = 0;
+        for (int t = t0; t < t1; ++t) {
+            const uint4 e = __ldg(reinterpret_cast<const uint4*>(T.zterms + t));
+            W pr = sext<W>((int64_t)(((uint64_t)e.y << 32) | e.x));
+            const int nf = (e.z >> 8) & 255;
+            const uint32_t w[2] = {e.z >> 16, e.w};
+#pragma unroll
+            for (int i = 0; i < 6; ++i) {      // constant shifts: no local memory
+                if (i >= nf) break;
+                const int code = i < 2 ? (int)((w[0] >> (8 * i)) & 255) : (int)((w[1] >> (8 * (i - 2))) & 255);
+                pr *= binom_fly<W>(zsel(z, code >> 5), code & 31);
+            }
+            sum += pr;
         }
+        bool o = false;
+        acc.v[p] = add_ovf(acc.v[p], (u128)sum, o);
+        if (o) acc.ovf |= 1u << p;
     }
-    W sum = 0;
-    int cur = -1;
-    for (int t = 0; t < T.zn; ++t) {
-        const ZTerm e = T.zterms[t];
-        if (e.pat != cur) {
-            if (cur >= 0) acc.add(cur, (u128)sum, false);
-            sum = 0;
-            cur = e.pat;
-        }
-        W pr = sext<W>(e.coef);
-        for (int i = 0; i < e.nf; ++i) pr *= R[e.f[i] * stride];
-        sum += pr;
-    }
-    if (cur >= 0) acc.add(cur, (u128)sum, false);
 }
 
 // Flush the warp's `cnt` buffered triangle matches (leaf[i * kLeafW + .]):
@@ -239,11 +257,12 @@ __device__ __noinline__ void tri_flush(const GraphDev& G, const HubDev& H, const
             lu = (int)L[0]; lv = (int)L[1]; lw = (int)L[2];
             du = (int)L[3]; dv = (int)L[4]; dw = (int)L[5];
             cuv = (int)L[6]; cvw = (int)L[8];
-            cuw = __ldg(sup + L[7]);
+            cuw = (int)L[7];
         }
         // leaves whose fc is 0 for every program (necessary condition from
         // degrees and supports) are counted as matches and skipped
-        const bool alive = mine && tri_alive(P, C, du, dv, dw, cuv, cuw, cvw);
+        // (the Z-term path without t evaluates every leaf: cheaper than the test)
+        const bool alive = mine && ((VD.zn && !VD.zneed7) || tri_alive(P, C, du, dv, dw, cuv, cuw, cvw));
         // Z-term path: tier bound from the largest Z in use and the largest
         // program (prod_t C(Z_t, k_t) <= Zmax^K); past 2^119 the leaf takes
         // the checked Listing 5 on its Venn diagram
@@ -294,9 +313,9 @@ __device__ __noinline__ void tri_flush(const GraphDev& G, const HubDev& H, const
             z[3] = cuv - 1; z[5] = cuw - 1; z[6] = cvw - 1;
             z[7] = t;
             if (alive && all64) {
-                zterms_eval<uint64_t>(z, VD, (uint64_t*)lane_rows, 2 * lane_stride, acc);
+                zterms_eval<uint64_t>(z, VD, acc);
             } else if (alive && !zfb) {
-                zterms_eval<u128>(z, VD, lane_rows, lane_stride, acc);
+                zterms_eval<u128>(z, VD, acc);
             }
             if (!__any_sync(FULLMASK, alive && zfb)) continue;
         }
@@ -365,13 +384,13 @@ __device__ __noinline__ void tri_flush(const GraphDev& G, const HubDev& H, const
 // append the hits of one round (hit: this lane's candidate c is in N+(b)) to
 // the warp's leaf buffer; the caller flushes at >= 32
 __device__ __forceinline__ int tri_append(uint32_t* leaf, int cnt, bool hit, int a, int b, int c, int du, int dv,
-                                          int dw, int cuv, uint32_t eac, int cvw, int lane) {
+                                          int dw, int cuv, int cuw, int cvw, int lane) {
     const unsigned fm = __ballot_sync(FULLMASK, hit);
     if (hit) {
         uint32_t* L = leaf + (cnt + __popc(fm & ((1u << lane) - 1))) * kLeafW;
         L[0] = (uint32_t)a; L[1] = (uint32_t)b; L[2] = (uint32_t)c;
         L[3] = (uint32_t)du; L[4] = (uint32_t)dv; L[5] = (uint32_t)dw;
-        L[6] = (uint32_t)cuv; L[7] = eac; L[8] = (uint32_t)cvw;
+        L[6] = (uint32_t)cuv; L[7] = (uint32_t)cuw; L[8] = (uint32_t)cvw;
     }
     return cnt + __popc(fm);
 }
@@ -495,14 +514,14 @@ __global__ void __launch_bounds__(kWarpTabWarps * 32) list_warp_kernel(
         const int total = carry;
         int lo = 0;                           // monotone: last j with pre[j] <= idx
         for (int v0 = 0; v0 < total; v0 += 64) {
-            int jj[2], cc[2];
+            int jj[2], cc[2], ca[2];
             uint32_t pp[2];
             bool ok[2];
 #pragma unroll
             for (int r = 0; r < 2; ++r) {
                 const int idx = v0 + 32 * r + lane;
                 ok[r] = idx < total;
-                jj[r] = 0; pp[r] = 0; cc[r] = -1;
+                jj[r] = 0; pp[r] = 0; cc[r] = -1; ca[r] = 0;
                 if (ok[r]) {
                     int l2 = lo, hi = len;
                     while (hi - l2 > 1) {
@@ -513,6 +532,7 @@ __global__ void __launch_bounds__(kWarpTabWarps * 32) list_warp_kernel(
                     jj[r] = l2;
                     pp[r] = q0[l2] + (uint32_t)(idx - pre[l2]);
                     cc[r] = __ldg(G.adj + pp[r]);
+                    if (TRI) ca[r] = __ldg(sup + (pp[r] - da[l2]));   // c(ac): coalesced along the tail
                 }
             }
 #pragma unroll
@@ -527,8 +547,8 @@ __global__ void __launch_bounds__(kWarpTabWarps * 32) list_warp_kernel(
                         cvw = pay0[kk];
                         if (W.degfilter && dw < C.mindeg2) hit = false;
                     }
-                    cnt = tri_append(leaf, cnt, hit, ea[jj[r]], b, cc[r], xa[jj[r]], degb, dw, ya[jj[r]],
-                                     pp[r] - da[jj[r]], cvw, lane);
+                    cnt = tri_append(leaf, cnt, hit, ea[jj[r]], b, cc[r], xa[jj[r]], degb, dw, ya[jj[r]], ca[r],
+                                     cvw, lane);
                     if (cnt >= 32) {
                         tri_flush<NP>(G, H, P, VD, C, sup, leaf, cnt, lrows, blockDim.x, wrows, lane, acc);
                         if (lane == 0) nmatch += cnt;
@@ -672,11 +692,12 @@ __global__ void __launch_bounds__((TRI ? kBlockTriWarps : kBlockTabWarps) * 32) 
                 }
                 int hits = 0;
                 for (int o0 = 0; o0 < Lt; o0 += 32 * kILP) {
-                    int cc[kILP];
+                    int cc[kILP], ca[kILP];
 #pragma unroll
                     for (int r = 0; r < kILP; ++r) {
                         const int o = o0 + 32 * r + lane;
                         cc[r] = o < Lt ? __ldg(G.adj + qt + o) : -1;
+                        ca[r] = (TRI && o < Lt) ? __ldg(sup + (qt + o - dt)) : 0;   // c(ac), coalesced
                     }
 #pragma unroll
                     for (int r = 0; r < kILP; ++r) {
@@ -691,8 +712,7 @@ __global__ void __launch_bounds__((TRI ? kBlockTriWarps : kBlockTabWarps) * 32) 
                                 cvw = pay0[kk];
                                 if (W.degfilter && dw < C.mindeg2) hit = false;
                             }
-                            cnt = tri_append(leaf, cnt, hit, at, b, cc[r], dat, degb, dw, cabt,
-                                             (uint32_t)(pos - dt), cvw, lane);
+                            cnt = tri_append(leaf, cnt, hit, at, b, cc[r], dat, degb, dw, cabt, ca[r], cvw, lane);
                             if (cnt >= 32) {
                                 tri_flush<NP>(G, H, P, VD, C, sup, leaf, cnt, lrows, nthr, wrows, lane, acc);
                                 if (lane == 0) nmatch += cnt;
