@@ -122,7 +122,8 @@ const void* np_kernel(int which, int np) {
     }
 }
 const void* kernel_for(int kind, int np) { return np_kernel(kind, np); }
-const void* tri_block_kernel(int np) { return np_kernel(4, np); }
+// triangle-core listing kernel: warp or block tables, every fc path or Z-only
+const void* tri_kernel(bool zonly, bool block, int np) { return np_kernel((zonly ? 5 : 3) + (block ? 1 : 0), np); }
 
 // hash bits of a block table holding out-degree `maxout` at load <= 1/2
 int table_hbits(int64_t maxout) {
@@ -244,6 +245,7 @@ struct PassExec {
     PassPlan plan;
     int kind = 0;              // 0 vertex, 1 edge (support + fc), 2 general core
     int npc = 1;               // accumulator width class
+    bool zonly = false;        // triangle cores: Z-term-only listing kernels (no leaf can leave the 128-bit tier)
     int64_t grid = 1;
     size_t smem = 0;
     WorkDesc W{};
@@ -593,11 +595,11 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
         if (g->sup_hash) {
             typedef WarpTabLayout<false> LS;
             P->grid_hash = std::max<int64_t>(1, std::min<int64_t>(
-                (int64_t)nsm * occupancy((const void*)list_warp_kernel<false, 1>, kWarpTabWarps * 32, LS::bytes),
+                (int64_t)nsm * occupancy((const void*)list_warp_kernel<0, 1>, kWarpTabWarps * 32, LS::bytes),
                 (g->nsup_units + kWarpTabWarps - 1) / kWarpTabWarps));
             P->hbits_big = table_hbits(g->sup_maxout);
             P->smem_big = blocktab_table_bytes(1 << P->hbits_big, (int)g->sup_maxout, false);
-            const int occ = occupancy((const void*)list_block_kernel<false, 1>, kBlockTabWarps * 32, P->smem_big);
+            const int occ = occupancy((const void*)list_block_kernel<0, 1>, kBlockTabWarps * 32, P->smem_big);
             if (g->nsup_units_big > 0 && occ == 0)
                 FSGC_FAIL(FSGC_ERR_INVALID, "block table of out-degree %lld does not fit shared memory",
                           (long long)g->sup_maxout);
@@ -720,7 +722,11 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
             // (the Z-term path keeps no rows: binomials are computed per factor)
             const size_t rows = X.vd.zn ? (size_t)0 : X.smem_vd;
             X.smem = WarpTabLayout<true>::bytes + rows;
-            int occ = occupancy(kernel_for(3, X.npc), kWarpTabWarps * 32, X.smem);
+            // Z-term-only kernels when the tier bound of the largest possible
+            // leaf (max degree) stays below the 128-bit limit of tri_flush
+            X.zonly = X.vd.zn > 0 && !tune("FSGC_NO_ZONLY", 0) &&
+                      (float)X.vd.zk * log2f((float)g->max_degree + 1.f) + X.vd.slack < 118.5f;
+            int occ = occupancy(tri_kernel(X.zonly, false, X.npc), kWarpTabWarps * 32, X.smem);
             if (occ == 0) FSGC_FAIL(FSGC_ERR_INVALID, "triangle-core pass: shared memory %zu B does not fit", X.smem);
             const int64_t units_w = (g->nsup_units + opts.shard_count - 1) / opts.shard_count;
             const int64_t units_b = (g->nsup_units_big + opts.shard_count - 1) / opts.shard_count;
@@ -729,7 +735,7 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
             X.hbits2 = table_hbits(g->sup_maxout);
             X.smem2 = blocktab_table_bytes(1 << X.hbits2, (int)g->sup_maxout, true) +
                       kBlockTriWarps * blocktab_warp_bytes(true) + rows;
-            occ = occupancy(tri_block_kernel(X.npc), kBlockTriWarps * 32, X.smem2);
+            occ = occupancy(tri_kernel(X.zonly, true, X.npc), kBlockTriWarps * 32, X.smem2);
             if (occ == 0 && units_b > 0)
                 FSGC_FAIL(FSGC_ERR_INVALID, "triangle-core pass: block table of out-degree %lld does not fit "
                           "shared memory (%zu B)", (long long)g->sup_maxout, X.smem2);
@@ -805,14 +811,14 @@ extern "C" int fsgc_plan_enqueue_stage(const fsgc_plan* P, void* workspace, void
                             (void*)&g->nsup_units_big, (void*)&hb, (void*)&mo, (void*)&dsup, (void*)&dq1,
                             (void*)&P->sup_shard, (void*)&P->sup_nshards, (void*)cp0, (void*)&W0, (void*)&V0,
                             (void*)&S0};
-            FSGC_CUDA(cudaLaunchKernel((const void*)list_block_kernel<false, 1>, dim3((unsigned)P->grid_hash_big),
+            FSGC_CUDA(cudaLaunchKernel((const void*)list_block_kernel<0, 1>, dim3((unsigned)P->grid_hash_big),
                                        dim3(kBlockTabWarps * 32), args, P->smem_big, st));
         }
         if (!merge_only && g->nsup_units > 0) {
             void* args[] = {(void*)&G, (void*)&O, (void*)&Hd, (void*)&g->rev, (void*)&g->sup_units,
                             (void*)&g->nsup_units, (void*)&dsup, (void*)&dq, (void*)&P->sup_shard,
                             (void*)&P->sup_nshards, (void*)cp0, (void*)&W0, (void*)&V0, (void*)&S0};
-            FSGC_CUDA(cudaLaunchKernel((const void*)list_warp_kernel<false, 1>, dim3((unsigned)P->grid_hash),
+            FSGC_CUDA(cudaLaunchKernel((const void*)list_warp_kernel<0, 1>, dim3((unsigned)P->grid_hash),
                                        dim3(kWarpTabWarps * 32), args, WarpTabLayout<false>::bytes, st));
         }
         if (merge_only) {
@@ -864,11 +870,11 @@ extern "C" int fsgc_plan_enqueue_stage(const fsgc_plan* P, void* workspace, void
                 FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(256), args_e, X.smem_fc, st));
             else if (X.kind == 3) {
                 if (g->nsup_units_big > 0)
-                    FSGC_CUDA(cudaLaunchKernel(tri_block_kernel(X.npc), dim3((unsigned)X.grid2),
+                    FSGC_CUDA(cudaLaunchKernel(tri_kernel(X.zonly, true, X.npc), dim3((unsigned)X.grid2),
                                                dim3(kBlockTriWarps * 32), args_t2, X.smem2, st));
                 if (g->nsup_units > 0)
-                    FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(kWarpTabWarps * 32), args_t, X.smem,
-                                               st));
+                    FSGC_CUDA(cudaLaunchKernel(tri_kernel(X.zonly, false, X.npc), dim3((unsigned)X.grid),
+                                               dim3(kWarpTabWarps * 32), args_t, X.smem, st));
             }
             else
                 FSGC_CUDA(cudaLaunchKernel(fn, dim3((unsigned)X.grid), dim3(kCoreWarps * 32), args_c,

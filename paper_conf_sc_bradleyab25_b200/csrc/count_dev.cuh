@@ -143,6 +143,16 @@ __device__ __forceinline__ void atomic_add_u128(AccDev* a, u128 v, bool ovf) {
     if (o) atomicOr(&a->ovf, 1u);
 }
 
+// One warp's pattern accumulators in SHARED memory (the triangle-core listing
+// kernels keep no per-lane register accumulators across the listing); lanes
+// may add concurrently, so the 128-bit add is two 64-bit atomics with carry.
+struct SAcc {
+    AccDev* a;   // [patterns]
+    __device__ __forceinline__ void add(int pat, u128 c, bool o) const {
+        if (c != 0 || o) atomic_add_u128(a + pat, c, o);
+    }
+};
+
 // Per-lane accumulators for NP patterns, register resident (pattern index
 // resolved by an unrolled compare, never by dynamic indexing).
 template <int NP>
@@ -765,9 +775,9 @@ __device__ __noinline__ float venn_bound_log2(const uint32_t* venn, int q, const
 // one diagram, every term of the pass, arithmetic mod 2^bits(W): exact when
 // each pattern's fc sum (>= every term, every partial sum) is below
 // 2^(bits - 9): then every used row entry C(n, s) and s * C(n, s) fit too
-template <class W, int NP>
+template <class W, class ACC>
 __device__ __forceinline__ void venn_terms_eval(const uint32_t* venn, int V, const VennDev& T, W* R, int stride,
-                                                AccN<NP>& acc) {
+                                                ACC& acc) {
     for (int r = 1; r < V; ++r) {      // R[base[r] + j - 1] = C(n_r, j), j = 1..maxs[r]
         const int K = T.maxs[r];
         if (!K) continue;
@@ -807,9 +817,9 @@ __device__ __forceinline__ void venn_terms_eval(const uint32_t* venn, int V, con
 // binomial row in the warp's shared buffer, then take the terms strided (each
 // lane's subsequence stays grouped by pattern, and its partial sums are
 // bounded by the pattern's sum, so the tier argument above holds per lane).
-template <class W, int NP>
+template <class W, class ACC>
 __device__ __forceinline__ void venn_warp_terms(const uint32_t* venn, int V, const VennDev& T, W* R, int lane,
-                                                AccN<NP>& acc) {
+                                                ACC& acc) {
     for (int r = 1 + lane; r < V; r += 32) {
         const int K = T.maxs[r];
         if (!K) continue;
@@ -876,9 +886,9 @@ __device__ __forceinline__ float venn_bound_log2_warp(const uint32_t* venn, int 
 
 // fc of one diagram by the whole warp: table tiers, else checked Listing 5
 // with the programs split over the lanes
-template <int STACK, int NP>
+template <int STACK, class ACC>
 __device__ __forceinline__ void venn_fc_warp(uint32_t* vloc, int q, const CoreProg& P, const VennDev& VD,
-                                             u128* rows, int lane, AccN<NP>& acc) {
+                                             u128* rows, int lane, ACC& acc) {
     const int V = 1 << q;
     const float bnd = venn_bound_log2_warp(vloc, q, P, lane) + VD.slack;
     if (bnd < 55.f) {

@@ -37,7 +37,7 @@
 //             function (Venn term table, else Listing 5).
 
 constexpr int kLeafCap = 64;      // leaf buffer per warp (flushed at >= 32)
-constexpr int kLeafW = 10;        // a, b, c, du, dv, dw, cuv, cuw, cvw, pad
+constexpr int kLeafW = 10;        // a, b, c, du, dv, dw, cuv, e(ac), cvw, pad
 constexpr int kILP = 4;           // tail loads in flight per lane (block tables)
 constexpr int kWarpTabWarps = 8;  // warps per block, warp-table kernels
 constexpr int kBlockTabWarps = 16;   // warps per block, block-table support kernel
@@ -179,12 +179,16 @@ __device__ __forceinline__ uint64_t sext<uint64_t>(int64_t c) { return (uint64_t
 template <>
 __device__ __forceinline__ u128 sext<u128>(int64_t c) { return (u128)(__int128)c; }
 
-// Z[cm] of one triangle leaf by core-position mask (registers, no dynamic
-// indexing: a select chain)
-__device__ __forceinline__ uint64_t zsel(const int (&z)[8], int cm) {
-    int r = z[1];
-#pragma unroll
-    for (int k = 2; k < 8; ++k) r = cm == k ? z[k] : r;
+// Z[cm] of one triangle leaf by core-position mask (a select chain: no
+// dynamic indexing)
+__device__ __forceinline__ uint64_t zsel(int z1, int z2, int z3, int z4, int z5, int z6, int z7, int cm) {
+    int r = z1;
+    r = cm == 2 ? z2 : r;
+    r = cm == 3 ? z3 : r;
+    r = cm == 4 ? z4 : r;
+    r = cm == 5 ? z5 : r;
+    r = cm == 6 ? z6 : r;
+    r = cm == 7 ? z7 : r;
     return (uint64_t)r;
 }
 
@@ -198,36 +202,46 @@ __device__ __forceinline__ W binom_fly(uint64_t n, int j) {
     return c;
 }
 
-// the Z-term table on one triangle (z[cm] = Z of the core-position set cm),
-// arithmetic mod 2^bits(W): exact when each pattern's sum over its programs
-// (a sum of products of binomials C(Z, k) bounded by the caller's bound) is
-// below 2^(bits - 9): then every binomial C(Z, j) fits with its 2-adic part.
-// Terms are grouped by pattern, so the accumulator index is static (the
-// pattern loop is unrolled) and no binomial rows are kept: each factor is
-// evaluated where it is used.
+// one pattern's terms [t0, t1) of the Z-term table on one triangle, mod
+// 2^bits(W).  Out of line: one copy per tier, called once per (leaf, pattern)
+template <class W>
+__device__ __noinline__ W zterm_sum(int z1, int z2, int z3, int z4, int z5, int z6, int z7, const ZTerm* __restrict__ zt,
+                                    int t0, int t1) {
+    W sum = 0;
+    for (int t = t0; t < t1; ++t) {
+        const uint4 e = __ldg(reinterpret_cast<const uint4*>(zt + t));
+        W pr = sext<W>((int64_t)(((uint64_t)e.y << 32) | e.x));
+        const int nf = (e.z >> 8) & 255;
+        uint64_t codes = (uint64_t)(e.z >> 16) | ((uint64_t)e.w << 16);   // 8-bit factor codes
+        for (int i = 0; i < nf; ++i, codes >>= 8) {
+            const int code = (int)(codes & 255);
+            pr *= binom_fly<W>(zsel(z1, z2, z3, z4, z5, z6, z7, code >> 5), code & 31);
+        }
+        sum += pr;
+    }
+    return sum;
+}
+
+// the Z-term table on the warp's 32 triangle leaves (z[cm] = Z of the
+// core-position set cm), arithmetic mod 2^bits(W): exact when each pattern's
+// sum over its programs (a sum of products of binomials C(Z, k) bounded by the
+// caller's bound) is below 2^(bits - 9): then every binomial C(Z, j) fits with
+// its 2-adic part.  Terms are grouped by pattern; each pattern's per-leaf sums
+// are reduced over the warp (shuffles) and lane 0 adds the total to the warp's
+// shared accumulator.  No binomial rows are kept.  Warp-uniform call.
 template <class W, int NP>
-__device__ __forceinline__ void zterms_eval(const int (&z)[8], const VennDev& T, AccN<NP>& acc) {
+__device__ __forceinline__ void zterms_eval_warp(bool act, const int (&z)[8], const VennDev& T, const SAcc& sa,
+                                                 int lane) {
 #pragma unroll
     for (int p = 0; p < NP; ++p) {
         const int t0 = T.zoff[p], t1 = T.zoff[p + 1];
         if (t0 == t1) continue;
-        W sum = 0;
-        for (int t = t0; t < t1; ++t) {
-            const uint4 e = __ldg(reinterpret_cast<const uint4*>(T.zterms + t));
-            W pr = sext<W>((int64_t)(((uint64_t)e.y << 32) | e.x));
-            const int nf = (e.z >> 8) & 255;
-            const uint32_t w[2] = {e.z >> 16, e.w};
-#pragma unroll
-            for (int i = 0; i < 6; ++i) {      // constant shifts: no local memory
-                if (i >= nf) break;
-                const int code = i < 2 ? (int)((w[0] >> (8 * i)) & 255) : (int)((w[1] >> (8 * (i - 2))) & 255);
-                pr *= binom_fly<W>(zsel(z, code >> 5), code & 31);
-            }
-            sum += pr;
-        }
+        W s = 0;
+        if (act) s = zterm_sum<W>(z[1], z[2], z[3], z[4], z[5], z[6], z[7], T.zterms, t0, t1);
+        u128 v = (u128)s;
         bool o = false;
-        acc.v[p] = add_ovf(acc.v[p], (u128)sum, o);
-        if (o) acc.ovf |= 1u << p;
+        warp_reduce_u128(v, o);
+        if (lane == 0 && (v != 0 || o)) atomic_add_u128(sa.a + p, v, o);
     }
 }
 
@@ -242,11 +256,14 @@ __device__ __forceinline__ void zterms_eval(const int (&z)[8], const VennDev& T,
 // N(u), the shortest list (u has the lowest degree), scanned against N(v),
 // N(w) through hub bitmaps or galloping cursors; warp-cooperative for long
 // lists.
-template <int NP>
+__device__ __noinline__ void tri_fc_venn(const CoreProg& P, const VennDev& VD, const TriCtx& C, bool alive, bool zfb,
+                                         int t, int du, int dv, int dw, int cuv, int cuw, int cvw, u128* lane_rows,
+                                         int lane_stride, u128* warp_rows, int lane, const SAcc acc);
+
+template <int NP, bool ZONLY>
 __device__ __noinline__ void tri_flush(const GraphDev& G, const HubDev& H, const CoreProg& P, const VennDev& VD,
                                        const TriCtx& C, const int* __restrict__ sup, uint32_t* leaf, int cnt,
-                                       u128* lane_rows, int lane_stride, u128* warp_rows, int lane,
-                                       AccN<NP>& acc) {
+                                       u128* lane_rows, int lane_stride, u128* warp_rows, int lane, const SAcc sa) {
     __syncwarp();
     for (int base = 0; base < cnt; base += 32) {
         const int li = base + lane;
@@ -257,7 +274,7 @@ __device__ __noinline__ void tri_flush(const GraphDev& G, const HubDev& H, const
             lu = (int)L[0]; lv = (int)L[1]; lw = (int)L[2];
             du = (int)L[3]; dv = (int)L[4]; dw = (int)L[5];
             cuv = (int)L[6]; cvw = (int)L[8];
-            cuw = (int)L[7];
+            cuw = __ldg(sup + L[7]);
         }
         // leaves whose fc is 0 for every program (necessary condition from
         // degrees and supports) are counted as matches and skipped
@@ -312,13 +329,22 @@ __device__ __noinline__ void tri_flush(const GraphDev& G, const HubDev& H, const
             z[1] = du - 2; z[2] = dv - 2; z[4] = dw - 2;
             z[3] = cuv - 1; z[5] = cuw - 1; z[6] = cvw - 1;
             z[7] = t;
-            if (alive && all64) {
-                zterms_eval<uint64_t>(z, VD, acc);
-            } else if (alive && !zfb) {
-                zterms_eval<u128>(z, VD, acc);
-            }
+            if (all64) zterms_eval_warp<uint64_t, NP>(alive, z, VD, sa, lane);
+            else zterms_eval_warp<u128, NP>(alive && !zfb, z, VD, sa, lane);
             if (!__any_sync(FULLMASK, alive && zfb)) continue;
         }
+        if constexpr (!ZONLY)
+            tri_fc_venn(P, VD, C, alive, zfb, t, du, dv, dw, cuv, cuw, cvw, lane_rows, lane_stride, warp_rows, lane,
+                        sa);
+    }
+    __syncwarp();
+}
+
+// the Venn-diagram part of the flush (out of line: not fetched on the Z-term
+// path): Venn term table (per lane or per warp), else checked Listing 5
+__device__ __noinline__ void tri_fc_venn(const CoreProg& P, const VennDev& VD, const TriCtx& C, bool alive, bool zfb,
+                                         int t, int du, int dv, int dw, int cuv, int cuw, int cvw, u128* lane_rows,
+                                         int lane_stride, u128* warp_rows, int lane, const SAcc acc) {
         uint32_t vq[8] = {0, 0, 0, 0, 0, 0, 0, 0};
         if (alive) {
             int R[8];
@@ -377,20 +403,35 @@ __device__ __noinline__ void tri_flush(const GraphDev& G, const HubDev& H, const
                     acc.add(fp.pat, f, o);
                 }
         }
-    }
+}
+
+// the warp's shared pattern sums as lane 0's register accumulators (for the
+// block reduction at the end of a kernel)
+template <int NP>
+__device__ __forceinline__ AccN<NP> sacc_to_lane0(const AccDev* a, int lane) {
     __syncwarp();
+    AccN<NP> A;
+    A.init();
+    if (lane == 0) {
+#pragma unroll
+        for (int p = 0; p < NP; ++p) {
+            A.v[p] = u128_make(a[p].lo, a[p].hi);
+            if (a[p].ovf) A.ovf |= 1u << p;
+        }
+    }
+    return A;
 }
 
 // append the hits of one round (hit: this lane's candidate c is in N+(b)) to
 // the warp's leaf buffer; the caller flushes at >= 32
 __device__ __forceinline__ int tri_append(uint32_t* leaf, int cnt, bool hit, int a, int b, int c, int du, int dv,
-                                          int dw, int cuv, int cuw, int cvw, int lane) {
+                                          int dw, int cuv, uint32_t eac, int cvw, int lane) {
     const unsigned fm = __ballot_sync(FULLMASK, hit);
     if (hit) {
         uint32_t* L = leaf + (cnt + __popc(fm & ((1u << lane) - 1))) * kLeafW;
         L[0] = (uint32_t)a; L[1] = (uint32_t)b; L[2] = (uint32_t)c;
         L[3] = (uint32_t)du; L[4] = (uint32_t)dv; L[5] = (uint32_t)dw;
-        L[6] = (uint32_t)cuv; L[7] = (uint32_t)cuw; L[8] = (uint32_t)cvw;
+        L[6] = (uint32_t)cuv; L[7] = eac; L[8] = (uint32_t)cvw;
     }
     return cnt + __popc(fm);
 }
@@ -411,11 +452,15 @@ struct WarpTabLayout {
     static constexpr size_t bytes = kWarpTabWarps * warp_b;
 };
 
-template <bool TRI, int NP>
+// MODE: 0 support pass, 1 triangle-core pass (every fc path), 2 triangle-core
+// pass on the Z-term path only (the host picks it when no leaf can leave the
+// 128-bit tier: no Venn / Listing 5 code in the kernel, fewer registers)
+template <int MODE, int NP>
 __global__ void __launch_bounds__(kWarpTabWarps * 32) list_warp_kernel(
     GraphDev G, OrientDev O, HubDev H, const int32_t* __restrict__ rev, const uint64_t* __restrict__ units,
     int64_t nunits, int* __restrict__ sup, unsigned long long* queue, int shard, int nshards, const __grid_constant__ CoreProg P,
     WorkDesc W, const __grid_constant__ VennDev VD, const Sink S) {
+    constexpr bool TRI = MODE != 0;
     typedef WarpTabLayout<TRI> Lay;
     extern __shared__ __align__(16) unsigned char s_lw[];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -435,8 +480,10 @@ __global__ void __launch_bounds__(kWarpTabWarps * 32) list_warp_kernel(
     u128* wrows = reinterpret_cast<u128*>(wb + Lay::slice_b + Lay::leaf_b);
     u128* lrows = reinterpret_cast<u128*>(s_lw + Lay::bytes) + threadIdx.x;  // lane-mode term rows
 
-    AccN<NP> acc;
-    acc.init();
+    __shared__ AccDev s_acc[kWarpTabWarps][TRI ? NP : 1];   // per-warp pattern sums (tri-core)
+    const SAcc sa{s_acc[w]};
+    if (TRI && lane < NP) s_acc[w][lane] = AccDev{0, 0, 0, 0, 0};
+    __syncwarp();
     unsigned long long nmatch = 0;
     TriCtx C;
     if (TRI) tri_ctx_init(C, P, W);
@@ -514,14 +561,14 @@ __global__ void __launch_bounds__(kWarpTabWarps * 32) list_warp_kernel(
         const int total = carry;
         int lo = 0;                           // monotone: last j with pre[j] <= idx
         for (int v0 = 0; v0 < total; v0 += 64) {
-            int jj[2], cc[2], ca[2];
+            int jj[2], cc[2];
             uint32_t pp[2];
             bool ok[2];
 #pragma unroll
             for (int r = 0; r < 2; ++r) {
                 const int idx = v0 + 32 * r + lane;
                 ok[r] = idx < total;
-                jj[r] = 0; pp[r] = 0; cc[r] = -1; ca[r] = 0;
+                jj[r] = 0; pp[r] = 0; cc[r] = -1;
                 if (ok[r]) {
                     int l2 = lo, hi = len;
                     while (hi - l2 > 1) {
@@ -532,7 +579,6 @@ __global__ void __launch_bounds__(kWarpTabWarps * 32) list_warp_kernel(
                     jj[r] = l2;
                     pp[r] = q0[l2] + (uint32_t)(idx - pre[l2]);
                     cc[r] = __ldg(G.adj + pp[r]);
-                    if (TRI) ca[r] = __ldg(sup + (pp[r] - da[l2]));   // c(ac): coalesced along the tail
                 }
             }
 #pragma unroll
@@ -547,10 +593,10 @@ __global__ void __launch_bounds__(kWarpTabWarps * 32) list_warp_kernel(
                         cvw = pay0[kk];
                         if (W.degfilter && dw < C.mindeg2) hit = false;
                     }
-                    cnt = tri_append(leaf, cnt, hit, ea[jj[r]], b, cc[r], xa[jj[r]], degb, dw, ya[jj[r]], ca[r],
-                                     cvw, lane);
+                    cnt = tri_append(leaf, cnt, hit, ea[jj[r]], b, cc[r], xa[jj[r]], degb, dw, ya[jj[r]],
+                                     pp[r] - da[jj[r]], cvw, lane);
                     if (cnt >= 32) {
-                        tri_flush<NP>(G, H, P, VD, C, sup, leaf, cnt, lrows, blockDim.x, wrows, lane, acc);
+                        tri_flush<NP, MODE == 2>(G, H, P, VD, C, sup, leaf, cnt, lrows, blockDim.x, wrows, lane, sa);
                         if (lane == 0) nmatch += cnt;
                         cnt = 0;
                     }
@@ -574,10 +620,10 @@ __global__ void __launch_bounds__(kWarpTabWarps * 32) list_warp_kernel(
     }
     if (TRI) {
         if (cnt) {
-            tri_flush<NP>(G, H, P, VD, C, sup, leaf, cnt, lrows, blockDim.x, wrows, lane, acc);
+            tri_flush<NP, MODE == 2>(G, H, P, VD, C, sup, leaf, cnt, lrows, blockDim.x, wrows, lane, sa);
             if (lane == 0) nmatch += cnt;
         }
-        block_publish<NP>(acc, nmatch, S);
+        block_publish<NP>(sacc_to_lane0<NP>(s_acc[w], lane), nmatch, S);
     } else if (prev_b >= 0) {
         __syncwarp();
         table_flush(O, sup, prev_b, hbits, key, kpos, pay0, lane, 32);
@@ -598,11 +644,12 @@ __host__ __device__ inline size_t blocktab_warp_bytes(bool tri) {
     return tri ? (size_t)kLeafCap * kLeafW * 4 + (size_t)kMaxVennRows * 16 : 0;
 }
 
-template <bool TRI, int NP>
-__global__ void __launch_bounds__((TRI ? kBlockTriWarps : kBlockTabWarps) * 32) list_block_kernel(
+template <int MODE, int NP>
+__global__ void __launch_bounds__((MODE ? kBlockTriWarps : kBlockTabWarps) * 32) list_block_kernel(
     GraphDev G, OrientDev O, HubDev H, const int32_t* __restrict__ rev, const uint64_t* __restrict__ units,
     int64_t nunits, int hbits_max, int maxout, int* __restrict__ sup, unsigned long long* queue, int shard, int nshards,
     const __grid_constant__ CoreProg P, WorkDesc W, const __grid_constant__ VennDev VD, const Sink S) {
+    constexpr bool TRI = MODE != 0;
     constexpr int NWB = TRI ? kBlockTriWarps : kBlockTabWarps;
     extern __shared__ __align__(16) unsigned char s_lb[];
     __shared__ long long s_unit;
@@ -619,8 +666,10 @@ __global__ void __launch_bounds__((TRI ? kBlockTriWarps : kBlockTabWarps) * 32) 
     u128* wrows = reinterpret_cast<u128*>(wb + (size_t)kLeafCap * kLeafW * 4);
     u128* lrows = reinterpret_cast<u128*>(s_lb + tab_b + NWB * blocktab_warp_bytes(TRI)) + tid;
 
-    AccN<NP> acc;
-    acc.init();
+    __shared__ AccDev s_acc[NWB][TRI ? NP : 1];   // per-warp pattern sums (tri-core)
+    const SAcc sa{s_acc[w]};
+    if (TRI && lane < NP) s_acc[w][lane] = AccDev{0, 0, 0, 0, 0};
+    __syncwarp();
     unsigned long long nmatch = 0;
     TriCtx C;
     if (TRI) tri_ctx_init(C, P, W);
@@ -692,12 +741,11 @@ __global__ void __launch_bounds__((TRI ? kBlockTriWarps : kBlockTabWarps) * 32) 
                 }
                 int hits = 0;
                 for (int o0 = 0; o0 < Lt; o0 += 32 * kILP) {
-                    int cc[kILP], ca[kILP];
+                    int cc[kILP];
 #pragma unroll
                     for (int r = 0; r < kILP; ++r) {
                         const int o = o0 + 32 * r + lane;
                         cc[r] = o < Lt ? __ldg(G.adj + qt + o) : -1;
-                        ca[r] = (TRI && o < Lt) ? __ldg(sup + (qt + o - dt)) : 0;   // c(ac), coalesced
                     }
 #pragma unroll
                     for (int r = 0; r < kILP; ++r) {
@@ -712,9 +760,10 @@ __global__ void __launch_bounds__((TRI ? kBlockTriWarps : kBlockTabWarps) * 32) 
                                 cvw = pay0[kk];
                                 if (W.degfilter && dw < C.mindeg2) hit = false;
                             }
-                            cnt = tri_append(leaf, cnt, hit, at, b, cc[r], dat, degb, dw, cabt, ca[r], cvw, lane);
+                            cnt = tri_append(leaf, cnt, hit, at, b, cc[r], dat, degb, dw, cabt,
+                                             (uint32_t)(pos - dt), cvw, lane);
                             if (cnt >= 32) {
-                                tri_flush<NP>(G, H, P, VD, C, sup, leaf, cnt, lrows, nthr, wrows, lane, acc);
+                                tri_flush<NP, MODE == 2>(G, H, P, VD, C, sup, leaf, cnt, lrows, nthr, wrows, lane, sa);
                                 if (lane == 0) nmatch += cnt;
                                 cnt = 0;
                             }
@@ -737,10 +786,10 @@ __global__ void __launch_bounds__((TRI ? kBlockTriWarps : kBlockTabWarps) * 32) 
     }
     if (TRI) {
         if (cnt) {
-            tri_flush<NP>(G, H, P, VD, C, sup, leaf, cnt, lrows, nthr, wrows, lane, acc);
+            tri_flush<NP, MODE == 2>(G, H, P, VD, C, sup, leaf, cnt, lrows, nthr, wrows, lane, sa);
             if (lane == 0) nmatch += cnt;
         }
-        block_publish<NP>(acc, nmatch, S);
+        block_publish<NP>(sacc_to_lane0<NP>(s_acc[w], lane), nmatch, S);
     } else if (cur_b >= 0) {
         table_flush(O, sup, cur_b, hbits, key, kpos, pay0, tid, nthr);
     }

@@ -5,7 +5,7 @@ TAG=$1; WL=$2; PATS=$3; KRE=${4:-list_}; CNT=${5:-4}
 OUT=gpurun_out
 TMP=/tmp/ncu_$TAG
 mkdir -p $TMP $OUT
-timeout 1500 ncu --set full --clock-control none --import-source on -k regex:$KRE -c $CNT \
+timeout 1500 ncu --set full --clock-control none --import-source on -k regex:$KRE -s ${SKIP:-0} -c $CNT \
   -o $TMP/prof -f python scripts/one_count.py $WL $PATS 1 > $OUT/ncu_${TAG}_${WL}.log 2>&1
 echo "ncu rc=$?"
 ncu -i $TMP/prof.ncu-rep --page raw --csv > $OUT/prof_${TAG}_${WL}_raw.csv 2>/dev/null
