@@ -447,6 +447,55 @@ static bool build_z_terms(const CoreProg& cp, const std::vector<std::vector<Part
     int progs_per_pat[FSGC_MAXPATS] = {0}, mp = 1;
     for (int pi = 0; pi < cp.nprog; ++pi) mp = std::max(mp, ++progs_per_pat[cp.prog[pi].pat]);
     hd->slack = std::log2((float)mp) + 2.f;
+    // tier thresholds on the leaf's largest degree (the device compares
+    // integers instead of evaluating the float bound per leaf)
+    auto tier_max = [&](float lim) {
+        int64_t lo = 0, hi = (int64_t)1 << 31;   // largest z with zk log2(z + 1) + slack < lim
+        if ((float)zk * log2f(1.f) + hd->slack >= lim) return (int32_t)-1;
+        while (hi - lo > 1) {
+            const int64_t mid = (lo + hi) / 2;
+            if ((float)zk * log2f((float)mid + 1.f) + hd->slack < lim) lo = mid; else hi = mid;
+        }
+        return (int32_t)std::min<int64_t>(lo, INT32_MAX);
+    };
+    hd->zmax64 = tier_max(55.f);
+    hd->zmax128 = tier_max(119.f);
+    // per pattern, the 64-bit tier of the row-free evaluation (arithmetic mod
+    // 2^64 is exact when (i) every binomial factor C(Z, j) times j fits -- the
+    // exact-division chain -- and (ii) the pattern's true per-leaf sum, which
+    // is at most sum_programs prod_t C(Z_t, k_t) <= #programs prod_t Z^k_t / k_t!,
+    // fits; partial sums and products may wrap, the ring arithmetic is exact
+    // mod 2^64).  Both in log2 with a 2-bit margin, Z <= the leaf's max degree.
+    {
+        double lfact[64];
+        lfact[0] = 0;
+        for (int j = 1; j < 64; ++j) lfact[j] = lfact[j - 1] + std::log2((double)j);
+        double nprog_p[FSGC_MAXPATS] = {0};
+        for (int pi = 0; pi < cp.nprog; ++pi) nprog_p[cp.prog[pi].pat] += 1;
+        for (int q = 0; q < FSGC_MAXPATS; ++q) {
+            auto fits = [&](double lz) {   // lz = log2(Z + 1)
+                double worst = 0;
+                for (int pi = 0; pi < cp.nprog; ++pi) {
+                    const FringeProg& fp = cp.prog[pi];
+                    if (fp.pat != q) continue;
+                    double b = 0;
+                    for (int t = 0; t < fp.s; ++t) {
+                        const int k = fp.k[t];
+                        b += k * lz - lfact[k];
+                        if (k * lz - lfact[k - 1] > 62.0) return false;   // C(Z, k) * k
+                    }
+                    worst = std::max(worst, b);
+                }
+                return worst + std::log2(std::max(1.0, nprog_p[q])) < 62.0;
+            };
+            int64_t lo = -1, hi = (int64_t)1 << 31;
+            while (hi - lo > 1) {
+                const int64_t mid = (lo + hi) / 2;
+                if (fits(std::log2((double)mid + 1.0))) lo = mid; else hi = mid;
+            }
+            hd->zmax64p[q] = (int32_t)std::min<int64_t>(lo, INT32_MAX);
+        }
+    }
     hd->zn = (int32_t)out->size();
     hd->znrows = nrows;
     hd->zneed7 = maxj[7] > 0;
@@ -673,6 +722,9 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
                     std::memcpy(hd.zmaxj, zh.zmaxj, 8);
                     std::memcpy(hd.zbase, zh.zbase, 8);
                     std::memcpy(hd.zoff, zh.zoff, sizeof hd.zoff);
+                    hd.zmax64 = zh.zmax64;
+                    std::memcpy(hd.zmax64p, zh.zmax64p, sizeof hd.zmax64p);
+                    hd.zmax128 = zh.zmax128;
                 } else {
                     zbase.push_back(0);
                 }
@@ -724,8 +776,7 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
             X.smem = WarpTabLayout<true>::bytes + rows;
             // Z-term-only kernels when the tier bound of the largest possible
             // leaf (max degree) stays below the 128-bit limit of tri_flush
-            X.zonly = X.vd.zn > 0 && !tune("FSGC_NO_ZONLY", 0) &&
-                      (float)X.vd.zk * log2f((float)g->max_degree + 1.f) + X.vd.slack < 118.5f;
+            X.zonly = X.vd.zn > 0 && !tune("FSGC_NO_ZONLY", 0) && g->max_degree <= X.vd.zmax128;
             int occ = occupancy(tri_kernel(X.zonly, false, X.npc), kWarpTabWarps * 32, X.smem);
             if (occ == 0) FSGC_FAIL(FSGC_ERR_INVALID, "triangle-core pass: shared memory %zu B does not fit", X.smem);
             const int64_t units_w = (g->nsup_units + opts.shard_count - 1) / opts.shard_count;

@@ -750,6 +750,10 @@ struct VennDev {
     uint8_t zmaxj[8];            // per core mask cm: max j of C(Z[cm], j)
     uint8_t zbase[8];            // per core mask cm: first row entry (unused by the row-free evaluation)
     uint16_t zoff[FSGC_MAXPATS + 1];   // terms of pattern p: [zoff[p], zoff[p+1]) (sorted by pattern)
+    int32_t zmax64, zmax128;     // largest max-degree of a leaf whose tier bound
+                                 // zk log2(Z + 1) + slack stays below 55 / 119
+    int32_t zmax64p[FSGC_MAXPATS];   // per pattern: largest leaf max-degree whose
+                                     // pattern sum and binomials fit 64 bits
 };
 
 // log2 upper bound of one pattern's fc sum on this diagram:

@@ -36,6 +36,9 @@
 //             through the Venn diagram (Sec. 3.3) and the fringe counting
 //             function (Venn term table, else Listing 5).
 
+#ifndef FSGC_ZONLY_MINB
+#define FSGC_ZONLY_MINB 4         // resident blocks per SM the Z-only listing kernels are compiled for
+#endif
 constexpr int kLeafCap = 64;      // leaf buffer per warp (flushed at >= 32)
 constexpr int kLeafW = 10;        // a, b, c, du, dv, dw, cuv, e(ac), cvw, pad
 constexpr int kILP = 4;           // tail loads in flight per lane (block tables)
@@ -223,22 +226,27 @@ __device__ __noinline__ W zterm_sum(int z1, int z2, int z3, int z4, int z5, int 
 }
 
 // the Z-term table on the warp's 32 triangle leaves (z[cm] = Z of the
-// core-position set cm), arithmetic mod 2^bits(W): exact when each pattern's
-// sum over its programs (a sum of products of binomials C(Z, k) bounded by the
-// caller's bound) is below 2^(bits - 9): then every binomial C(Z, j) fits with
-// its 2-adic part.  Terms are grouped by pattern; each pattern's per-leaf sums
+// core-position set cm), arithmetic mod 2^64 or 2^128 per pattern (the host's
+// per-pattern threshold on the leaf's largest degree: the binomials times j
+// and the pattern's per-leaf sum fit 64 bits; else 128 bits, which the
+// kernel's global bound guarantees).  Terms are grouped by pattern; each pattern's per-leaf sums
 // are reduced over the warp (shuffles) and lane 0 adds the total to the warp's
 // shared accumulator.  No binomial rows are kept.  Warp-uniform call.
-template <class W, int NP>
-__device__ __forceinline__ void zterms_eval_warp(bool act, const int (&z)[8], const VennDev& T, const SAcc& sa,
-                                                 int lane) {
+template <int NP>
+__device__ __forceinline__ void zterms_eval_warp(bool act, int zmax, const int (&z)[8], const VennDev& T,
+                                                 const SAcc& sa, int lane) {
 #pragma unroll
     for (int p = 0; p < NP; ++p) {
         const int t0 = T.zoff[p], t1 = T.zoff[p + 1];
         if (t0 == t1) continue;
-        W s = 0;
-        if (act) s = zterm_sum<W>(z[1], z[2], z[3], z[4], z[5], z[6], z[7], T.zterms, t0, t1);
-        u128 v = (u128)s;
+        // the tier per pattern (warp-uniform): 64-bit unless some leaf's
+        // largest degree exceeds the pattern's 64-bit threshold
+        u128 v = 0;
+        if (__all_sync(FULLMASK, !act || zmax <= T.zmax64p[p])) {
+            if (act) v = (u128)zterm_sum<uint64_t>(z[1], z[2], z[3], z[4], z[5], z[6], z[7], T.zterms, t0, t1);
+        } else {
+            if (act) v = zterm_sum<u128>(z[1], z[2], z[3], z[4], z[5], z[6], z[7], T.zterms, t0, t1);
+        }
         bool o = false;
         warp_reduce_u128(v, o);
         if (lane == 0 && (v != 0 || o)) atomic_add_u128(sa.a + p, v, o);
@@ -283,12 +291,8 @@ __device__ __noinline__ void tri_flush(const GraphDev& G, const HubDev& H, const
         // Z-term path: tier bound from the largest Z in use and the largest
         // program (prod_t C(Z_t, k_t) <= Zmax^K); past 2^119 the leaf takes
         // the checked Listing 5 on its Venn diagram
-        float zb = 0.f;
-        if (VD.zn && alive) {
-            const int zmax = max(max(du, dv), dw);
-            zb = (float)VD.zk * log2f((float)zmax + 1.f) + VD.slack;
-        }
-        const bool zfb = VD.zn && zb >= 119.f;
+        const int zmax = max(max(du, dv), dw);   // >= every Z of the leaf
+        const bool zfb = !ZONLY && VD.zn && alive && zmax > VD.zmax128;
         const bool want_t = alive && (VD.zn ? (VD.zneed7 || (zfb && C.need_t)) : C.need_t);
         const bool heavy = want_t && du > 32;
         if (want_t && !heavy) {
@@ -323,14 +327,12 @@ __device__ __noinline__ void tri_flush(const GraphDev& G, const HubDev& H, const
             t = max(max(0, cuv + cuw - du), max(cuv + cvw - dv, cuw + cvw - dw));
         }
         if (VD.zn) {                   // fc from the Z values (no Venn diagram)
-            const bool all64 = __all_sync(FULLMASK, !alive || zb < 55.f);
             int z[8];
             z[0] = 0;
             z[1] = du - 2; z[2] = dv - 2; z[4] = dw - 2;
             z[3] = cuv - 1; z[5] = cuw - 1; z[6] = cvw - 1;
             z[7] = t;
-            if (all64) zterms_eval_warp<uint64_t, NP>(alive, z, VD, sa, lane);
-            else zterms_eval_warp<u128, NP>(alive && !zfb, z, VD, sa, lane);
+            zterms_eval_warp<NP>(alive && !zfb, zmax, z, VD, sa, lane);
             if (!__any_sync(FULLMASK, alive && zfb)) continue;
         }
         if constexpr (!ZONLY)
@@ -456,7 +458,7 @@ struct WarpTabLayout {
 // pass on the Z-term path only (the host picks it when no leaf can leave the
 // 128-bit tier: no Venn / Listing 5 code in the kernel, fewer registers)
 template <int MODE, int NP>
-__global__ void __launch_bounds__(kWarpTabWarps * 32) list_warp_kernel(
+__global__ void __launch_bounds__(kWarpTabWarps * 32, MODE == 2 ? FSGC_ZONLY_MINB : 1) list_warp_kernel(
     GraphDev G, OrientDev O, HubDev H, const int32_t* __restrict__ rev, const uint64_t* __restrict__ units,
     int64_t nunits, int* __restrict__ sup, unsigned long long* queue, int shard, int nshards, const __grid_constant__ CoreProg P,
     WorkDesc W, const __grid_constant__ VennDev VD, const Sink S) {
@@ -645,7 +647,8 @@ __host__ __device__ inline size_t blocktab_warp_bytes(bool tri) {
 }
 
 template <int MODE, int NP>
-__global__ void __launch_bounds__((MODE ? kBlockTriWarps : kBlockTabWarps) * 32) list_block_kernel(
+__global__ void __launch_bounds__((MODE ? kBlockTriWarps : kBlockTabWarps) * 32, MODE == 2 ? FSGC_ZONLY_MINB : 1)
+    list_block_kernel(
     GraphDev G, OrientDev O, HubDev H, const int32_t* __restrict__ rev, const uint64_t* __restrict__ units,
     int64_t nunits, int hbits_max, int maxout, int* __restrict__ sup, unsigned long long* queue, int shard, int nshards,
     const __grid_constant__ CoreProg P, WorkDesc W, const __grid_constant__ VennDev VD, const Sink S) {

@@ -27,3 +27,15 @@ print(f"# {path}: {len(data)} rows, total samples {tot:.0f}; columns: {h[:12]}")
 data.sort(key=lambda x: -x[0])
 for v, r in data[:top]:
     print(f"{100 * v / tot:6.2f}%  " + " | ".join(x.strip()[:90] for x in r[:4]))
+
+# all rows as (offset from the function's first instruction, samples, warp
+# instructions executed) for local mapping to source lines (nvdisasm -g)
+if len(sys.argv) > 3:
+    addr = [int(r[col["Address"]], 16) for _, r in data]
+    base = min(addr) if addr else 0
+    ie = col.get("Instructions Executed")
+    with open(sys.argv[3], "w") as f:
+        for (v, r), a in zip(data, addr):
+            x = r[ie].replace(",", "") if ie is not None else "0"
+            if v or (x not in ("", "0")):
+                f.write(f"{a - base},{v:.0f},{x}\n")
