@@ -45,6 +45,7 @@ constexpr int kILP = 4;           // tail loads in flight per lane (block tables
 constexpr int kWarpTabWarps = 8;  // warps per block, warp-table kernels
 constexpr int kBlockTabWarps = 16;   // warps per block, block-table support kernel
 constexpr int kBlockTriWarps = 8;    // warps per block, block-table tri-core kernel
+constexpr int kSubC = 512;           // in-entries per concatenated sub-chunk, block-table kernels
 
 __device__ __forceinline__ uint32_t hslot(int x, int hbits) { return ((uint32_t)x * 0x9E3779B1u) >> (32 - hbits); }
 
@@ -208,11 +209,11 @@ __device__ __forceinline__ W binom_fly(uint64_t n, int j) {
 // one pattern's terms [t0, t1) of the Z-term table on one triangle, mod
 // 2^bits(W).  Out of line: one copy per tier, called once per (leaf, pattern)
 template <class W>
-__device__ __noinline__ W zterm_sum(int z1, int z2, int z3, int z4, int z5, int z6, int z7, const ZTerm* __restrict__ zt,
+__device__ __noinline__ W zterm_sum(int z1, int z2, int z3, int z4, int z5, int z6, int z7, const ZTerm* zt,
                                     int t0, int t1) {
     W sum = 0;
     for (int t = t0; t < t1; ++t) {
-        const uint4 e = __ldg(reinterpret_cast<const uint4*>(zt + t));
+        const uint4 e = *reinterpret_cast<const uint4*>(zt + t);   // shared (staged) or global
         W pr = sext<W>((int64_t)(((uint64_t)e.y << 32) | e.x));
         const int nf = (e.z >> 8) & 255;
         uint64_t codes = (uint64_t)(e.z >> 16) | ((uint64_t)e.w << 16);   // 8-bit factor codes
@@ -232,24 +233,51 @@ __device__ __noinline__ W zterm_sum(int z1, int z2, int z3, int z4, int z5, int 
 // kernel's global bound guarantees).  Terms are grouped by pattern; each pattern's per-leaf sums
 // are reduced over the warp (shuffles) and lane 0 adds the total to the warp's
 // shared accumulator.  No binomial rows are kept.  Warp-uniform call.
-template <int NP>
-__device__ __forceinline__ void zterms_eval_warp(bool act, int zmax, const int (&z)[8], const VennDev& T,
-                                                 const SAcc& sa, int lane) {
+// the pass's Z-term table staged in shared memory at kernel start (the flush
+// is out of line, so reading it from the kernel parameters would go through
+// generic loads)
+constexpr int kZShared = 128;
+struct ZShared {
+    const ZTerm* terms;          // shared copy (or the global table when it is larger)
+    const uint16_t* zoff;        // [FSGC_MAXPATS + 1]
+    const int32_t* z64;          // [FSGC_MAXPATS]
+};
+
+// warp sum of a non-negative value below 2^(16 * limbs): the 16-bit limbs
+// are summed with __reduce_add_sync (each limb sum < 2^21), then recombined --
+// a handful of REDUX instead of a 5-round 128-bit shuffle tree
+template <int LIMBS>
+__device__ __forceinline__ u128 warp_sum_limbs(u128 v) {
+    u128 tot = 0;
 #pragma unroll
+    for (int l = 0; l < LIMBS; ++l) {
+        const unsigned part = __reduce_add_sync(FULLMASK, (unsigned)((uint64_t)(v >> (16 * l)) & 0xffffu));
+        tot += (u128)part << (16 * l);
+    }
+    return tot;
+}
+
+template <int NP>
+__device__ __forceinline__ void zterms_eval_warp(bool act, int zmax, const int (&z)[8], const ZShared& T,
+                                                 const SAcc& sa, int lane) {
+    // (a runtime pattern loop: the accumulators are in shared memory, so the
+    // code is not replicated per pattern)
+#pragma unroll 1
     for (int p = 0; p < NP; ++p) {
         const int t0 = T.zoff[p], t1 = T.zoff[p + 1];
         if (t0 == t1) continue;
         // the tier per pattern (warp-uniform): 64-bit unless some leaf's
-        // largest degree exceeds the pattern's 64-bit threshold
-        u128 v = 0;
-        if (__all_sync(FULLMASK, !act || zmax <= T.zmax64p[p])) {
-            if (act) v = (u128)zterm_sum<uint64_t>(z[1], z[2], z[3], z[4], z[5], z[6], z[7], T.zterms, t0, t1);
+        // largest degree exceeds the pattern's 64-bit threshold (then the
+        // per-leaf sum is below 2^119 by the kernel's bound)
+        u128 tot;
+        if (__all_sync(FULLMASK, !act || zmax <= T.z64[p])) {
+            const uint64_t v = act ? zterm_sum<uint64_t>(z[1], z[2], z[3], z[4], z[5], z[6], z[7], T.terms, t0, t1) : 0;
+            tot = warp_sum_limbs<4>((u128)v);      // 32 x < 2^62: the sum fits 67 bits
         } else {
-            if (act) v = zterm_sum<u128>(z[1], z[2], z[3], z[4], z[5], z[6], z[7], T.zterms, t0, t1);
+            const u128 v = act ? zterm_sum<u128>(z[1], z[2], z[3], z[4], z[5], z[6], z[7], T.terms, t0, t1) : 0;
+            tot = warp_sum_limbs<8>(v);            // 32 x < 2^119 < 2^128
         }
-        bool o = false;
-        warp_reduce_u128(v, o);
-        if (lane == 0 && (v != 0 || o)) atomic_add_u128(sa.a + p, v, o);
+        if (lane == 0 && tot != 0) atomic_add_u128(sa.a + p, tot, false);
     }
 }
 
@@ -271,7 +299,8 @@ __device__ __noinline__ void tri_fc_venn(const CoreProg& P, const VennDev& VD, c
 template <int NP, bool ZONLY>
 __device__ __noinline__ void tri_flush(const GraphDev& G, const HubDev& H, const CoreProg& P, const VennDev& VD,
                                        const TriCtx& C, const int* __restrict__ sup, uint32_t* leaf, int cnt,
-                                       u128* lane_rows, int lane_stride, u128* warp_rows, int lane, const SAcc sa) {
+                                       u128* lane_rows, int lane_stride, u128* warp_rows, int lane, const SAcc sa,
+                                       const ZShared ZS) {
     __syncwarp();
     for (int base = 0; base < cnt; base += 32) {
         const int li = base + lane;
@@ -332,7 +361,7 @@ __device__ __noinline__ void tri_flush(const GraphDev& G, const HubDev& H, const
             z[1] = du - 2; z[2] = dv - 2; z[4] = dw - 2;
             z[3] = cuv - 1; z[5] = cuw - 1; z[6] = cvw - 1;
             z[7] = t;
-            zterms_eval_warp<NP>(alive && !zfb, zmax, z, VD, sa, lane);
+            zterms_eval_warp<NP>(alive && !zfb, zmax, z, ZS, sa, lane);
             if (!__any_sync(FULLMASK, alive && zfb)) continue;
         }
         if constexpr (!ZONLY)
@@ -407,6 +436,18 @@ __device__ __noinline__ void tri_fc_venn(const CoreProg& P, const VennDev& VD, c
         }
 }
 
+// stage the Z-term table of the pass in shared memory (block-wide, the caller
+// synchronises)
+__device__ __forceinline__ ZShared zshared_stage(const VennDev& VD, ZTerm* s_zt, uint16_t* s_zoff, int32_t* s_z64,
+                                                 int tid, int nthr) {
+    const bool fits = VD.zn <= kZShared;
+    if (fits)
+        for (int i = tid; i < VD.zn; i += nthr) s_zt[i] = VD.zterms[i];
+    for (int i = tid; i <= FSGC_MAXPATS; i += nthr) s_zoff[i] = VD.zoff[i];
+    for (int i = tid; i < FSGC_MAXPATS; i += nthr) s_z64[i] = VD.zmax64p[i];
+    return ZShared{fits ? s_zt : VD.zterms, s_zoff, s_z64};
+}
+
 // the warp's shared pattern sums as lane 0's register accumulators (for the
 // block reduction at the end of a kernel)
 template <int NP>
@@ -458,7 +499,7 @@ struct WarpTabLayout {
 // pass on the Z-term path only (the host picks it when no leaf can leave the
 // 128-bit tier: no Venn / Listing 5 code in the kernel, fewer registers)
 template <int MODE, int NP>
-__global__ void __launch_bounds__(kWarpTabWarps * 32, MODE == 2 ? FSGC_ZONLY_MINB : 1) list_warp_kernel(
+__global__ void __launch_bounds__(kWarpTabWarps * 32, MODE == 2 ? FSGC_ZONLY_MINB : MODE + 1) list_warp_kernel(
     GraphDev G, OrientDev O, HubDev H, const int32_t* __restrict__ rev, const uint64_t* __restrict__ units,
     int64_t nunits, int* __restrict__ sup, unsigned long long* queue, int shard, int nshards, const __grid_constant__ CoreProg P,
     WorkDesc W, const __grid_constant__ VennDev VD, const Sink S) {
@@ -483,9 +524,14 @@ __global__ void __launch_bounds__(kWarpTabWarps * 32, MODE == 2 ? FSGC_ZONLY_MIN
     u128* lrows = reinterpret_cast<u128*>(s_lw + Lay::bytes) + threadIdx.x;  // lane-mode term rows
 
     __shared__ AccDev s_acc[kWarpTabWarps][TRI ? NP : 1];   // per-warp pattern sums (tri-core)
+    __shared__ ZTerm s_zt[TRI ? kZShared : 1];
+    __shared__ uint16_t s_zoff[FSGC_MAXPATS + 1];
+    __shared__ int32_t s_z64[FSGC_MAXPATS];
     const SAcc sa{s_acc[w]};
     if (TRI && lane < NP) s_acc[w][lane] = AccDev{0, 0, 0, 0, 0};
-    __syncwarp();
+    ZShared ZS{nullptr, nullptr, nullptr};
+    if (TRI) ZS = zshared_stage(VD, s_zt, s_zoff, s_z64, threadIdx.x, blockDim.x);
+    __syncthreads();
     unsigned long long nmatch = 0;
     TriCtx C;
     if (TRI) tri_ctx_init(C, P, W);
@@ -598,7 +644,7 @@ __global__ void __launch_bounds__(kWarpTabWarps * 32, MODE == 2 ? FSGC_ZONLY_MIN
                     cnt = tri_append(leaf, cnt, hit, ea[jj[r]], b, cc[r], xa[jj[r]], degb, dw, ya[jj[r]],
                                      pp[r] - da[jj[r]], cvw, lane);
                     if (cnt >= 32) {
-                        tri_flush<NP, MODE == 2>(G, H, P, VD, C, sup, leaf, cnt, lrows, blockDim.x, wrows, lane, sa);
+                        tri_flush<NP, MODE == 2>(G, H, P, VD, C, sup, leaf, cnt, lrows, blockDim.x, wrows, lane, sa, ZS);
                         if (lane == 0) nmatch += cnt;
                         cnt = 0;
                     }
@@ -622,7 +668,7 @@ __global__ void __launch_bounds__(kWarpTabWarps * 32, MODE == 2 ? FSGC_ZONLY_MIN
     }
     if (TRI) {
         if (cnt) {
-            tri_flush<NP, MODE == 2>(G, H, P, VD, C, sup, leaf, cnt, lrows, blockDim.x, wrows, lane, sa);
+            tri_flush<NP, MODE == 2>(G, H, P, VD, C, sup, leaf, cnt, lrows, blockDim.x, wrows, lane, sa, ZS);
             if (lane == 0) nmatch += cnt;
         }
         block_publish<NP>(sacc_to_lane0<NP>(s_acc[w], lane), nmatch, S);
@@ -647,7 +693,7 @@ __host__ __device__ inline size_t blocktab_warp_bytes(bool tri) {
 }
 
 template <int MODE, int NP>
-__global__ void __launch_bounds__((MODE ? kBlockTriWarps : kBlockTabWarps) * 32, MODE == 2 ? FSGC_ZONLY_MINB : 1)
+__global__ void __launch_bounds__((MODE ? kBlockTriWarps : kBlockTabWarps) * 32, MODE == 2 ? FSGC_ZONLY_MINB : MODE)
     list_block_kernel(
     GraphDev G, OrientDev O, HubDev H, const int32_t* __restrict__ rev, const uint64_t* __restrict__ units,
     int64_t nunits, int hbits_max, int maxout, int* __restrict__ sup, unsigned long long* queue, int shard, int nshards,
@@ -657,6 +703,11 @@ __global__ void __launch_bounds__((MODE ? kBlockTriWarps : kBlockTabWarps) * 32,
     extern __shared__ __align__(16) unsigned char s_lb[];
     __shared__ long long s_unit;
     __shared__ int s_next;
+    __shared__ int32_t s_pre[kSubC + 1];          // sub-chunk: exclusive scan of the tail lengths
+    __shared__ uint32_t s_q0[kSubC], s_da[kSubC];  // tail start in adj, split[a] - oofs[a]
+    __shared__ int32_t s_e[kSubC], s_x[kSubC];     // support: e(ab), c(ab) count | tri-core: a, deg a
+    __shared__ int32_t s_y[TRI ? kSubC : 1];       // tri-core: c(ab)
+    __shared__ int32_t s_wsum[NWB];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, tid = threadIdx.x, nthr = blockDim.x;
     const int HS = 1 << hbits_max;
     const size_t tab_b = blocktab_table_bytes(HS, maxout, TRI);
@@ -670,9 +721,14 @@ __global__ void __launch_bounds__((MODE ? kBlockTriWarps : kBlockTabWarps) * 32,
     u128* lrows = reinterpret_cast<u128*>(s_lb + tab_b + NWB * blocktab_warp_bytes(TRI)) + tid;
 
     __shared__ AccDev s_acc[NWB][TRI ? NP : 1];   // per-warp pattern sums (tri-core)
+    __shared__ ZTerm s_zt[TRI ? kZShared : 1];
+    __shared__ uint16_t s_zoff[FSGC_MAXPATS + 1];
+    __shared__ int32_t s_z64[FSGC_MAXPATS];
     const SAcc sa{s_acc[w]};
     if (TRI && lane < NP) s_acc[w][lane] = AccDev{0, 0, 0, 0, 0};
-    __syncwarp();
+    ZShared ZS{nullptr, nullptr, nullptr};
+    if (TRI) ZS = zshared_stage(VD, s_zt, s_zoff, s_z64, tid, nthr);
+    __syncthreads();
     unsigned long long nmatch = 0;
     TriCtx C;
     if (TRI) tri_ctx_init(C, P, W);
@@ -709,87 +765,133 @@ __global__ void __launch_bounds__((MODE ? kBlockTriWarps : kBlockTabWarps) * 32,
         const int64_t ib0 = __ldg(G.offs + b) + (int64_t)k * FSGC_SUP_CHUNK;
         const int len = skip ? 0 : (int)min((int64_t)FSGC_SUP_CHUNK, sb - ib0);
         const int64_t rbase = ib0 - __ldg(O.oofs + b);
-        for (;;) {
-            int j0 = 0;
-            if (lane == 0) j0 = atomicAdd(&s_next, 32);
-            j0 = __shfl_sync(FULLMASK, j0, 0);
-            if (j0 >= len) break;
-            const int j = j0 + lane;
-            int64_t qa = 0, dA = 0;
-            int La = 0, e = 0, a = 0, dga = 0, cab = 0;
-            if (j < len) {
-                a = __ldg(G.adj + ib0 + j);
-                e = __ldg(rev + rbase + j);
-                const int64_t sa = __ldg(O.split + a), oa = __ldg(O.oofs + a);
-                qa = sa + (e - oa) + 1;
-                La = (int)(__ldg(G.offs + a + 1) - qa);
-                dA = sa - oa;
-                if (TRI) {
-                    dga = (int)(__ldg(G.offs + a + 1) - __ldg(G.offs + a));
-                    cab = __ldg(sup + e);
-                    if ((W.degfilter && dga < C.mindeg0) || cab == 0) La = 0;
-                }
-            }
-            const int nj = min(32, len - j0);
-            for (int tt = 0; tt < nj; ++tt) {
-                const int Lt = __shfl_sync(FULLMASK, La, tt);
-                if (Lt == 0) continue;
-                const int64_t qt = __shfl_sync(FULLMASK, qa, tt);
-                const int64_t dt = __shfl_sync(FULLMASK, dA, tt);
-                int at = 0, dat = 0, cabt = 0;
-                if (TRI) {
-                    at = __shfl_sync(FULLMASK, a, tt);
-                    dat = __shfl_sync(FULLMASK, dga, tt);
-                    cabt = __shfl_sync(FULLMASK, cab, tt);
-                }
-                int hits = 0;
-                for (int o0 = 0; o0 < Lt; o0 += 32 * kILP) {
-                    int cc[kILP];
-#pragma unroll
-                    for (int r = 0; r < kILP; ++r) {
-                        const int o = o0 + 32 * r + lane;
-                        cc[r] = o < Lt ? __ldg(G.adj + qt + o) : -1;
+        // the unit in sub-chunks of kSubC in-entries; per sub-chunk the tails
+        // are concatenated (block-wide exclusive scan of their lengths) and
+        // the warps take 32 * kILP consecutive virtual elements at a time: the
+        // work is balanced within the block whatever the tail lengths (the
+        // heavy middles' tails are mostly short), and every lane has an
+        // element each step
+        for (int sc = 0; sc < len; sc += kSubC) {
+            const int sl = min(kSubC, len - sc);
+            for (int j = tid; j < kSubC; j += nthr) {
+                int L = 0;
+                if (j < sl) {
+                    const int a = __ldg(G.adj + ib0 + sc + j);
+                    const int e = __ldg(rev + rbase + sc + j);
+                    const int64_t sa_ = __ldg(O.split + a), oa = __ldg(O.oofs + a);
+                    const int64_t q = sa_ + (e - oa) + 1;
+                    const int64_t ea = __ldg(G.offs + a + 1);
+                    L = (int)(ea - q);
+                    s_q0[j] = (uint32_t)q;
+                    s_da[j] = (uint32_t)(sa_ - oa);
+                    if (TRI) {
+                        const int dga = (int)(ea - __ldg(G.offs + a));
+                        const int cab = __ldg(sup + e);
+                        s_e[j] = a;
+                        s_x[j] = dga;
+                        s_y[j] = cab;
+                        if ((W.degfilter && dga < C.mindeg0) || cab == 0) L = 0;   // no triangle on (a, b)
+                    } else {
+                        s_e[j] = e;
+                        s_x[j] = 0;
                     }
+                }
+                s_pre[j] = L;
+            }
+            if (tid == 0) s_next = 0;
+            __syncthreads();
+            {   // exclusive scan of s_pre[0, kSubC): a segment per warp, then the warp offsets
+                constexpr int segL = kSubC / NWB;
+                int run = 0;
+                for (int c0 = 0; c0 < segL; c0 += 32) {
+                    const int j = w * segL + c0 + lane;
+                    const int v = s_pre[j];
+                    int x = v;
 #pragma unroll
-                    for (int r = 0; r < kILP; ++r) {
-                        const int h = cc[r] >= 0 ? hfind(key, cc[r], hbits) : -1;
-                        bool hit = h >= 0;
-                        const int64_t pos = qt + o0 + 32 * r + lane;
-                        if (TRI) {
-                            int dw = 0, cvw = 0;
-                            if (hit) {
-                                const int kk = kpos[h];
-                                dw = pay1[kk];
-                                cvw = pay0[kk];
-                                if (W.degfilter && dw < C.mindeg2) hit = false;
-                            }
-                            cnt = tri_append(leaf, cnt, hit, at, b, cc[r], dat, degb, dw, cabt,
-                                             (uint32_t)(pos - dt), cvw, lane);
-                            if (cnt >= 32) {
-                                tri_flush<NP, MODE == 2>(G, H, P, VD, C, sup, leaf, cnt, lrows, nthr, wrows, lane, sa);
-                                if (lane == 0) nmatch += cnt;
-                                cnt = 0;
-                            }
-                        } else {
-                            if (hit) {
-                                atomicAdd(&pay0[h], 1);                  // c(bc)
-                                atomicAdd(sup + (pos - dt), 1);          // c(ac)
-                            }
-                            hits += __popc(__ballot_sync(FULLMASK, hit));
+                    for (int o = 1; o < 32; o <<= 1) {
+                        const int y = __shfl_up_sync(FULLMASK, x, o);
+                        if (lane >= o) x += y;
+                    }
+                    s_pre[j] = run + x - v;
+                    run += __shfl_sync(FULLMASK, x, 31);
+                }
+                if (lane == 0) s_wsum[w] = run;
+                __syncthreads();
+                int off = 0;
+                for (int q = 0; q < w; ++q) off += s_wsum[q];
+                for (int c0 = 0; c0 < segL; c0 += 32) s_pre[w * segL + c0 + lane] += off;
+                if (w == NWB - 1 && lane == 0) s_pre[kSubC] = off + run;
+                __syncthreads();
+            }
+            const int total = s_pre[kSubC];
+            int lo = 0;                        // per lane: monotone over its elements
+            for (;;) {
+                int e0 = 0;
+                if (lane == 0) e0 = atomicAdd(&s_next, 32 * kILP);
+                e0 = __shfl_sync(FULLMASK, e0, 0);
+                if (e0 >= total) break;
+                int jj[kILP], cc[kILP];
+                uint32_t pp[kILP];
+#pragma unroll
+                for (int r = 0; r < kILP; ++r) {   // last j with pre[j] <= idx: a non-empty tail
+                    const int idx = e0 + 32 * r + lane;
+                    jj[r] = 0; pp[r] = 0; cc[r] = -1;
+                    if (idx < total) {
+                        int l2 = lo, hi = kSubC;
+                        if (s_pre[l2] > idx) l2 = 0;
+                        while (hi - l2 > 1) {
+                            const int mid = (l2 + hi) >> 1;
+                            if (s_pre[mid] <= idx) l2 = mid; else hi = mid;
+                        }
+                        lo = l2;
+                        jj[r] = l2;
+                        pp[r] = s_q0[l2] + (uint32_t)(idx - s_pre[l2]);
+                        cc[r] = __ldg(G.adj + pp[r]);
+                    }
+                }
+#pragma unroll
+                for (int r = 0; r < kILP; ++r) {
+                    const int h = cc[r] >= 0 ? hfind(key, cc[r], hbits) : -1;
+                    bool hit = h >= 0;
+                    const int j = jj[r];
+                    if (TRI) {
+                        int dw = 0, cvw = 0;
+                        if (hit) {
+                            const int kk = kpos[h];
+                            dw = pay1[kk];
+                            cvw = pay0[kk];
+                            if (W.degfilter && dw < C.mindeg2) hit = false;
+                        }
+                        cnt = tri_append(leaf, cnt, hit, s_e[j], b, cc[r], s_x[j], degb, dw, s_y[j],
+                                         pp[r] - s_da[j], cvw, lane);
+                        if (cnt >= 32) {
+                            tri_flush<NP, MODE == 2>(G, H, P, VD, C, sup, leaf, cnt, lrows, nthr, wrows, lane, sa, ZS);
+                            if (lane == 0) nmatch += cnt;
+                            cnt = 0;
+                        }
+                    } else {
+                        const unsigned hmask = __ballot_sync(FULLMASK, hit);
+                        if (hit) {
+                            atomicAdd(&pay0[h], 1);                        // c(bc)
+                            atomicAdd(sup + (pp[r] - s_da[j]), 1);          // c(ac)
+                            const unsigned peers = __match_any_sync(hmask, j);   // c(ab): one add per a
+                            if ((peers & ((1u << lane) - 1)) == 0) atomicAdd(&s_x[j], __popc(peers));
                         }
                     }
                 }
-                if (!TRI) {
-                    const int et = __shfl_sync(FULLMASK, e, tt);
-                    if (lane == 0 && hits) atomicAdd(sup + et, hits);   // c(ab)
-                }
+            }
+            __syncthreads();
+            if (!TRI) {
+                for (int j = tid; j < sl; j += nthr)
+                    if (s_x[j]) atomicAdd(sup + s_e[j], s_x[j]);
+                __syncthreads();
             }
         }
         __syncthreads();
     }
     if (TRI) {
         if (cnt) {
-            tri_flush<NP, MODE == 2>(G, H, P, VD, C, sup, leaf, cnt, lrows, nthr, wrows, lane, sa);
+            tri_flush<NP, MODE == 2>(G, H, P, VD, C, sup, leaf, cnt, lrows, nthr, wrows, lane, sa, ZS);
             if (lane == 0) nmatch += cnt;
         }
         block_publish<NP>(sacc_to_lane0<NP>(s_acc[w], lane), nmatch, S);

@@ -479,6 +479,33 @@ def test_k_tailed_triangles_rmat16_closed_form(sup_mode):
         assert F.fsgc_count(g, [pats[k - 1]])[0].count == want, k
 
 
+def test_triangle_core_z_tiers_hub_closed_form(sup_mode):
+    """Triangle core forced (configs[4] patterns) on a hub of degree 200k whose
+    triangles mix with hub-free ones: the row-free Z-term path evaluates each
+    pattern in 64 or 128 bits by the per-pattern threshold on the leaf's
+    largest degree (4-tailed: 128-bit for hub leaves, 3-tailed and below:
+    64-bit), so both tiers and both tier choices meet in one warp.  Every
+    k-tailed triangle/tricore count equals the closed form sum over triangles
+    of C(deg x - 2, k) (oracle.k_tailed_triangles, pinned), and the triangle
+    count the plain listing."""
+    import numpy as np
+    rng = np.random.default_rng(11)
+    H = 200_000
+    hub = np.stack([np.zeros(H, np.int64), np.arange(1, H + 1)], 1)
+    leaf = rng.integers(1, 20_001, size=(6000, 2))
+    extra = rng.integers(H + 1, H + 3001, size=(20000, 2))   # a hub-free dense-ish part
+    e = np.concatenate([hub, leaf, extra])
+    n = H + 3001
+    offs, adj, _ = oracle.degree_ordered_csr(n, e)
+    gadj = oracle.csr_to_adjacency(offs, adj)
+    g = F.fsgc_load_graph(e, n)
+    names = ["triangle/tricore", "tricore+1f"] + [f"{k}-tailed-triangle/tricore" for k in (2, 3, 4)]
+    res = F.fsgc_count(g, [F.compile_named(PATTERNS[x]) for x in names])
+    want = [oracle.k_tailed_triangles(gadj, 0) // 3] + [oracle.k_tailed_triangles(gadj, k) for k in (1, 2, 3, 4)]
+    for x, r, w in zip(names, res, want):
+        assert not r.overflow and r.count == w, (x, r.count, w)
+
+
 @pytest.mark.parametrize("wl", ["rmat16", "pl2k"])
 def test_wedge_hash_support_equals_merge(wl, monkeypatch):
     """The support pass's two algorithms -- the wedge-hash kernels (middle
