@@ -147,6 +147,15 @@ def measured_peaks():
     return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
 
 
+def ncu_r02(workload):
+    """per-kernel ncu numbers of this round's capture (profiles/ncu_r02_summary.json,
+    written by scripts/ncu_r02_summary.py from an ncu run of the same build)"""
+    path = os.path.join(ROOT, "profiles", "ncu_r02_summary.json")
+    if not os.path.exists(path):
+        return {}
+    return json.load(open(path)).get(workload, {}).get("kernels", {})
+
+
 def ncu_traffic(workload, kernel):
     """dram__bytes_read + dram__bytes_write per launch of `kernel` from the
     committed `ncu --set full` summary (profiles/ncu_summary.json), or None."""
@@ -565,20 +574,49 @@ def main():
             byts = 8.0 * (n + 1) * share
         else:   # compulsory graph bytes: CSR + oriented view + supports, read once
             byts = (8.0 * 2 * m + 8.0 * (n + 1) + 8.0 * m + 4.0 * m + 16.0 * n) * share
-        kernels.append((names[kind] + f" [pass {k}]", byts, kms_sum[k] / args.steps))
+        kernels.append((names[kind] + f" [pass {k}]", byts, kms_sum[k] / args.steps, kind))
         if kind != 0 and ams_sum[k] > 0:
             kernels.append((("list_*_kernel<support> (per-edge |N(u)&N(v)|, listing by middle vertex)"
                              if hash_mode else "support_kernel (per-edge |N(u)&N(v)|, merge)") + f" [pass {k}]",
-                            sup_b, ams_sum[k] / args.steps))
+                            sup_b, ams_sum[k] / args.steps, "support"))
     kernels.sort(key=lambda kk: -kk[2])
     peak, peak_src = measured_peaks()
+    nsm = torch.cuda.get_device_properties(dev).multi_processor_count
+    ncu = ncu_r02(args.workload)
 
-    def roof(name, byts, ms):
-        traffic = ncu_traffic(graph_key(args.workload), name)
-        ach = byts / (ms / 1e3) / 1e9 if ms > 0 else 0.0
-        return {"bound": "hbm", "achieved": ach, "peak": peak, "unit": "GB/s", "frac": ach / peak,
-                "traffic": traffic, "kernel": name, "kernel_ms": ms, "share_of_step": ms / ms_per_step,
-                "algorithmic_bytes_per_launch": byts, "peak_source": peak_src}
+    def ncu_sum(prefixes, field):
+        vals = [v.get(field) for k, v in ncu.items() if any(k.startswith(p) for p in prefixes)]
+        vals = [x for x in vals if x is not None]
+        return sum(vals) if vals else None
+
+    def roof(name, byts, ms, kind):
+        hbm_ach = byts / (ms / 1e3) / 1e9 if ms > 0 else 0.0
+        if kind == "support":
+            traffic = ncu_sum(("list_block_kernel<support>", "list_warp_kernel<support>", "support_kernel"),
+                              "dram_bytes_per_launch")
+        elif kind == 3:
+            traffic = ncu_sum(("list_block_kernel<tri", "list_warp_kernel<tri"), "dram_bytes_per_launch")
+        else:
+            traffic = ncu_traffic(graph_key(args.workload), name)
+        out = {"bound": "hbm", "achieved": hbm_ach, "peak": peak, "unit": "GB/s", "frac": hbm_ach / peak,
+               "traffic": traffic, "kernel": name, "kernel_ms": ms, "share_of_step": ms / ms_per_step,
+               "algorithmic_bytes_per_launch": byts, "peak_source": peak_src}
+        inst = ncu_sum(("list_block_kernel<tri", "list_warp_kernel<tri"), "inst_per_launch") if kind == 3 else None
+        if inst and ms > 0 and clocks.get("sm_mhz"):
+            # the triangle-core pass is bound by instruction issue (fc
+            # arithmetic + listing), not by bytes: DESIGN.md Sec. 5 -- warp
+            # instructions of the pass (ncu, same build and workload) per
+            # second of the live-timed pass, against SMs x 4 schedulers x 1
+            # warp-instruction / clock at the sampled SM clock
+            ipk = nsm * 4 * clocks["sm_mhz"] * 1e6
+            ach = inst * share / (ms / 1e3)
+            out = {"bound": "alu", "achieved": ach, "peak": ipk, "unit": "warp-inst/s", "frac": ach / ipk,
+                   "traffic": traffic, "kernel": name, "kernel_ms": ms, "share_of_step": ms / ms_per_step,
+                   "inst_per_launch": inst * share, "peak_source": f"{nsm} SMs x 4 issue slots x {clocks['sm_mhz']} MHz "
+                                                                 "(sampled under load)",
+                   "hbm_view": {"algorithmic_bytes_per_launch": byts, "achieved_gbs": hbm_ach, "peak_gbs": peak,
+                                "frac": hbm_ach / peak}}
+        return out
 
     # ---- e2e through the public API from pinned host buffers
     e2e = None

@@ -642,7 +642,7 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
     }
     if (P->sup_first >= 0) {
         if (g->sup_hash) {
-            typedef WarpTabLayout<false> LS;
+            typedef WarpTabLayout<0> LS;
             P->grid_hash = std::max<int64_t>(1, std::min<int64_t>(
                 (int64_t)nsm * occupancy((const void*)list_warp_kernel<0, 1>, kWarpTabWarps * 32, LS::bytes),
                 (g->nsup_units + kWarpTabWarps - 1) / kWarpTabWarps));
@@ -773,10 +773,10 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
             // lane-mode term rows (kTriWarps * 32 threads): Venn table and/or Z table
             // (the Z-term path keeps no rows: binomials are computed per factor)
             const size_t rows = X.vd.zn ? (size_t)0 : X.smem_vd;
-            X.smem = WarpTabLayout<true>::bytes + rows;
             // Z-term-only kernels when the tier bound of the largest possible
             // leaf (max degree) stays below the 128-bit limit of tri_flush
             X.zonly = X.vd.zn > 0 && !tune("FSGC_NO_ZONLY", 0) && g->max_degree <= X.vd.zmax128;
+            X.smem = (X.zonly ? WarpTabLayout<2>::bytes : WarpTabLayout<1>::bytes) + rows;
             int occ = occupancy(tri_kernel(X.zonly, false, X.npc), kWarpTabWarps * 32, X.smem);
             if (occ == 0) FSGC_FAIL(FSGC_ERR_INVALID, "triangle-core pass: shared memory %zu B does not fit", X.smem);
             const int64_t units_w = (g->nsup_units + opts.shard_count - 1) / opts.shard_count;
@@ -785,13 +785,17 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
                                                             (units_w + kWarpTabWarps - 1) / kWarpTabWarps));
             X.hbits2 = table_hbits(g->sup_maxout);
             X.smem2 = blocktab_table_bytes(1 << X.hbits2, (int)g->sup_maxout, true) +
-                      kBlockTriWarps * blocktab_warp_bytes(true) + rows;
+                      kBlockTriWarps * blocktab_warp_bytes(X.zonly ? 2 : 1) + rows;
             occ = occupancy(tri_kernel(X.zonly, true, X.npc), kBlockTriWarps * 32, X.smem2);
             if (occ == 0 && units_b > 0)
                 FSGC_FAIL(FSGC_ERR_INVALID, "triangle-core pass: block table of out-degree %lld does not fit "
                           "shared memory (%zu B)", (long long)g->sup_maxout, X.smem2);
             X.grid2 = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * std::max(1, std::min(occ, 16)) ,
                                                              std::max<int64_t>(1, units_b)));
+            if (tune("FSGC_VENN_INFO", 0))
+                fprintf(stderr, "[tri] zonly %d; warp tables: %zu B smem, grid %lld; block tables (max out %lld): "
+                        "%zu B smem, %d blocks/SM, grid %lld\n", (int)X.zonly, X.smem, (long long)X.grid,
+                        (long long)g->sup_maxout, X.smem2, occ, (long long)X.grid2);
             if (X.grid + X.grid2 > (int64_t)nsm * 16)
                 FSGC_FAIL(FSGC_ERR_INTERNAL, "triangle-core pass: block partials overflow");
         }
@@ -870,7 +874,7 @@ extern "C" int fsgc_plan_enqueue_stage(const fsgc_plan* P, void* workspace, void
                             (void*)&g->nsup_units, (void*)&dsup, (void*)&dq, (void*)&P->sup_shard,
                             (void*)&P->sup_nshards, (void*)cp0, (void*)&W0, (void*)&V0, (void*)&S0};
             FSGC_CUDA(cudaLaunchKernel((const void*)list_warp_kernel<0, 1>, dim3((unsigned)P->grid_hash),
-                                       dim3(kWarpTabWarps * 32), args, WarpTabLayout<false>::bytes, st));
+                                       dim3(kWarpTabWarps * 32), args, WarpTabLayout<0>::bytes, st));
         }
         if (merge_only) {
             support_kernel<<<(int)P->grid_sup, 256, 0, st>>>(G, O, g->nsup_merge, dsup, g->sorder, g->ssrc, g->sdst,

@@ -45,7 +45,8 @@ constexpr int kILP = 4;           // tail loads in flight per lane (block tables
 constexpr int kWarpTabWarps = 8;  // warps per block, warp-table kernels
 constexpr int kBlockTabWarps = 16;   // warps per block, block-table support kernel
 constexpr int kBlockTriWarps = 8;    // warps per block, block-table tri-core kernel
-constexpr int kSubC = 512;           // in-entries per concatenated sub-chunk, block-table kernels
+constexpr int kSubCSup = 512;        // in-entries per concatenated sub-chunk, block-table support kernel
+constexpr int kSubCTri = 256;        // ... tri-core kernel (shared memory: 2 blocks/SM with RMAT-26's table)
 
 __device__ __forceinline__ uint32_t hslot(int x, int hbits) { return ((uint32_t)x * 0x9E3779B1u) >> (32 - hbits); }
 
@@ -257,7 +258,7 @@ __device__ __forceinline__ u128 warp_sum_limbs(u128 v) {
     return tot;
 }
 
-template <int NP>
+template <int NP, bool ZONLY>
 __device__ __forceinline__ void zterms_eval_warp(bool act, int zmax, const int (&z)[8], const ZShared& T,
                                                  const SAcc& sa, int lane) {
     // (a runtime pattern loop: the accumulators are in shared memory, so the
@@ -277,7 +278,18 @@ __device__ __forceinline__ void zterms_eval_warp(bool act, int zmax, const int (
             const u128 v = act ? zterm_sum<u128>(z[1], z[2], z[3], z[4], z[5], z[6], z[7], T.terms, t0, t1) : 0;
             tot = warp_sum_limbs<8>(v);            // 32 x < 2^119 < 2^128
         }
-        if (lane == 0 && tot != 0) atomic_add_u128(sa.a + p, tot, false);
+        if (lane == 0 && tot != 0) {
+            if (ZONLY) {   // only this lane writes the warp's sums: a plain 128-bit add
+                AccDev& d = sa.a[p];
+                const u128 old = u128_make(d.lo, d.hi);
+                const u128 nw = old + tot;
+                d.lo = u128_lo(nw);
+                d.hi = u128_hi(nw);
+                if (nw < old) d.ovf = 1;
+            } else {       // the Venn / Listing 5 lanes of this warp add atomically
+                atomic_add_u128(sa.a + p, tot, false);
+            }
+        }
     }
 }
 
@@ -361,7 +373,7 @@ __device__ __noinline__ void tri_flush(const GraphDev& G, const HubDev& H, const
             z[1] = du - 2; z[2] = dv - 2; z[4] = dw - 2;
             z[3] = cuv - 1; z[5] = cuw - 1; z[6] = cvw - 1;
             z[7] = t;
-            zterms_eval_warp<NP>(alive && !zfb, zmax, z, ZS, sa, lane);
+            zterms_eval_warp<NP, ZONLY>(alive && !zfb, zmax, z, ZS, sa, lane);
             if (!__any_sync(FULLMASK, alive && zfb)) continue;
         }
         if constexpr (!ZONLY)
@@ -482,15 +494,17 @@ __device__ __forceinline__ int tri_append(uint32_t* leaf, int cnt, bool hit, int
 // ------------------------------------------------------------------------
 // warp-table kernel.  Shared memory per warp: table (key, kpos/cnt or
 // tsup/tdeg: HS = 2 * FSGC_SUP_CAPW slots), slice arrays, leaf buffer (TRI)
-template <bool TRI>
+constexpr int kWSub = 64;    // in-entries per half-slice of a warp unit (FSGC_SUP_SEG = 2 halves)
+template <int MODE>
 struct WarpTabLayout {
+    static constexpr bool TRI = MODE != 0;
     static constexpr int HS = 2 * FSGC_SUP_CAPW;
     static constexpr size_t key_b = (size_t)HS * 4;
     static constexpr size_t kpos_b = (size_t)HS * 2;
     static constexpr size_t pay_b = TRI ? (size_t)FSGC_SUP_CAPW * 8 : (size_t)HS * 4;   // tsup+tdeg | cnt
-    static constexpr size_t slice_b = (size_t)(FSGC_SUP_SEG + 4) * 4 + (size_t)5 * FSGC_SUP_SEG * 4;
+    static constexpr size_t slice_b = (size_t)(kWSub + 4) * 4 + (size_t)5 * kWSub * 4;
     static constexpr size_t leaf_b = TRI ? (size_t)kLeafCap * kLeafW * 4 : 0;
-    static constexpr size_t rows_b = TRI ? (size_t)kMaxVennRows * 16 : 0;     // warp-mode term rows
+    static constexpr size_t rows_b = MODE == 1 ? (size_t)kMaxVennRows * 16 : 0;     // warp-mode term rows
     static constexpr size_t warp_b = key_b + kpos_b + pay_b + slice_b + leaf_b + rows_b;
     static constexpr size_t bytes = kWarpTabWarps * warp_b;
 };
@@ -504,7 +518,7 @@ __global__ void __launch_bounds__(kWarpTabWarps * 32, MODE == 2 ? FSGC_ZONLY_MIN
     int64_t nunits, int* __restrict__ sup, unsigned long long* queue, int shard, int nshards, const __grid_constant__ CoreProg P,
     WorkDesc W, const __grid_constant__ VennDev VD, const Sink S) {
     constexpr bool TRI = MODE != 0;
-    typedef WarpTabLayout<TRI> Lay;
+    typedef WarpTabLayout<MODE> Lay;
     extern __shared__ __align__(16) unsigned char s_lw[];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
     unsigned char* tb = s_lw + (size_t)w * Lay::warp_b;
@@ -513,12 +527,12 @@ __global__ void __launch_bounds__(kWarpTabWarps * 32, MODE == 2 ? FSGC_ZONLY_MIN
     int32_t* pay0 = reinterpret_cast<int32_t*>(tb + Lay::key_b + Lay::kpos_b);   // cnt[slot] | tsup[pos]
     int32_t* pay1 = pay0 + FSGC_SUP_CAPW;                                         // - | tdeg[pos]
     unsigned char* wb = tb + Lay::key_b + Lay::kpos_b + Lay::pay_b;
-    int32_t* pre = reinterpret_cast<int32_t*>(wb);                           // [SEG + 4]
-    uint32_t* q0 = reinterpret_cast<uint32_t*>(wb + (FSGC_SUP_SEG + 4) * 4);  // tail start per in-entry
-    uint32_t* da = q0 + FSGC_SUP_SEG;                                        // split[a] - oofs[a]
-    int32_t* ea = reinterpret_cast<int32_t*>(da + FSGC_SUP_SEG);             // e(ab) | a
-    int32_t* xa = ea + FSGC_SUP_SEG;                                         // c(ab) count | deg a
-    int32_t* ya = xa + FSGC_SUP_SEG;                                         // - | c(ab)
+    int32_t* pre = reinterpret_cast<int32_t*>(wb);                           // [kWSub + 4]
+    uint32_t* q0 = reinterpret_cast<uint32_t*>(wb + (kWSub + 4) * 4);        // tail start per in-entry
+    uint32_t* da = q0 + kWSub;                                               // split[a] - oofs[a]
+    int32_t* ea = reinterpret_cast<int32_t*>(da + kWSub);                    // e(ab) | a
+    int32_t* xa = ea + kWSub;                                                // c(ab) count | deg a
+    int32_t* ya = xa + kWSub;                                                // - | c(ab)
     uint32_t* leaf = reinterpret_cast<uint32_t*>(wb + Lay::slice_b);
     u128* wrows = reinterpret_cast<u128*>(wb + Lay::slice_b + Lay::leaf_b);
     u128* lrows = reinterpret_cast<u128*>(s_lw + Lay::bytes) + threadIdx.x;  // lane-mode term rows
@@ -566,105 +580,111 @@ __global__ void __launch_bounds__(kWarpTabWarps * 32, MODE == 2 ? FSGC_ZONLY_MIN
             __syncwarp();
         }
         if (TRI && W.degfilter && degb < C.mindeg1) continue;
-        const int64_t ib0 = __ldg(G.offs + b) + (int64_t)k * FSGC_SUP_SEG;
-        const int len = (int)min((int64_t)FSGC_SUP_SEG, sb - ib0);
-        const int64_t rbase = ib0 - __ldg(O.oofs + b);
-        // slice setup: per in-entry a the start q0 of its tail (after b in
-        // N+(a)) and the tail length; exclusive scan of the lengths -> pre
-        int carry = 0;
-        for (int j0 = 0; j0 < len; j0 += 32) {
-            const int j = j0 + lane;
-            int Lt = 0;
-            if (j < len) {
-                const int a = __ldg(G.adj + ib0 + j);
-                const int e = __ldg(rev + rbase + j);
-                const int64_t sa = __ldg(O.split + a), oa = __ldg(O.oofs + a);
-                const int64_t q = sa + (e - oa) + 1;
-                Lt = (int)(__ldg(G.offs + a + 1) - q);
-                q0[j] = (uint32_t)q;
-                da[j] = (uint32_t)(sa - oa);
-                if (TRI) {
-                    const int dga = (int)(__ldg(G.offs + a + 1) - __ldg(G.offs + a));
-                    ea[j] = a;
-                    xa[j] = dga;
-                    ya[j] = __ldg(sup + e);
-                    if (W.degfilter && dga < C.mindeg0) Lt = 0;
-                    if (ya[j] == 0) Lt = 0;          // no triangle on (a, b)
-                } else {
-                    ea[j] = e;
-                    xa[j] = 0;
-                }
-            }
-            int x = Lt;                       // inclusive warp scan
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const int y = __shfl_up_sync(FULLMASK, x, o);
-                if (lane >= o) x += y;
-            }
-            if (j < len) pre[j] = carry + x - Lt;
-            carry += __shfl_sync(FULLMASK, x, 31);
-        }
-        if (lane == 0) pre[len] = carry;
-        __syncwarp();
-        const int total = carry;
-        int lo = 0;                           // monotone: last j with pre[j] <= idx
-        for (int v0 = 0; v0 < total; v0 += 64) {
-            int jj[2], cc[2];
-            uint32_t pp[2];
-            bool ok[2];
-#pragma unroll
-            for (int r = 0; r < 2; ++r) {
-                const int idx = v0 + 32 * r + lane;
-                ok[r] = idx < total;
-                jj[r] = 0; pp[r] = 0; cc[r] = -1;
-                if (ok[r]) {
-                    int l2 = lo, hi = len;
-                    while (hi - l2 > 1) {
-                        const int mid = (l2 + hi) >> 1;
-                        if (pre[mid] <= idx) l2 = mid; else hi = mid;
-                    }
-                    lo = l2;
-                    jj[r] = l2;
-                    pp[r] = q0[l2] + (uint32_t)(idx - pre[l2]);
-                    cc[r] = __ldg(G.adj + pp[r]);
-                }
-            }
-#pragma unroll
-            for (int r = 0; r < 2; ++r) {
-                const int h = ok[r] ? hfind(key, cc[r], hbits) : -1;
-                bool hit = h >= 0;
-                if (TRI) {
-                    int dw = 0, cvw = 0;
-                    if (hit) {
-                        const int kk = kpos[h];
-                        dw = pay1[kk];
-                        cvw = pay0[kk];
-                        if (W.degfilter && dw < C.mindeg2) hit = false;
-                    }
-                    cnt = tri_append(leaf, cnt, hit, ea[jj[r]], b, cc[r], xa[jj[r]], degb, dw, ya[jj[r]],
-                                     pp[r] - da[jj[r]], cvw, lane);
-                    if (cnt >= 32) {
-                        tri_flush<NP, MODE == 2>(G, H, P, VD, C, sup, leaf, cnt, lrows, blockDim.x, wrows, lane, sa, ZS);
-                        if (lane == 0) nmatch += cnt;
-                        cnt = 0;
-                    }
-                } else {
-                    const unsigned hmask = __ballot_sync(FULLMASK, hit);
-                    if (hit) {
-                        atomicAdd(&pay0[h], 1);                              // c(bc)
-                        atomicAdd(sup + (pp[r] - da[jj[r]]), 1);             // c(ac)
-                        const unsigned peers = __match_any_sync(hmask, jj[r]);   // c(ab): one add per a
-                        if ((peers & ((1u << lane) - 1)) == 0) atomicAdd(&xa[jj[r]], __popc(peers));
+        // the unit's FSGC_SUP_SEG in-entries in halves of kWSub (half the
+        // slice arrays in shared memory per warp: more resident warps)
+        const int64_t ibu = __ldg(G.offs + b) + (int64_t)k * FSGC_SUP_SEG;
+        const int lenu = (int)min((int64_t)FSGC_SUP_SEG, sb - ibu);
+        for (int h0 = 0; h0 < lenu; h0 += kWSub) {
+            const int64_t ib0 = ibu + h0;
+            const int len = min(kWSub, lenu - h0);
+            const int64_t rbase = ib0 - __ldg(O.oofs + b);
+            // slice setup: per in-entry a the start q0 of its tail (after b in
+            // N+(a)) and the tail length; exclusive scan of the lengths -> pre
+            int carry = 0;
+            for (int j0 = 0; j0 < len; j0 += 32) {
+                const int j = j0 + lane;
+                int Lt = 0;
+                if (j < len) {
+                    const int a = __ldg(G.adj + ib0 + j);
+                    const int e = __ldg(rev + rbase + j);
+                    const int64_t sa = __ldg(O.split + a), oa = __ldg(O.oofs + a);
+                    const int64_t q = sa + (e - oa) + 1;
+                    Lt = (int)(__ldg(G.offs + a + 1) - q);
+                    q0[j] = (uint32_t)q;
+                    da[j] = (uint32_t)(sa - oa);
+                    if (TRI) {
+                        const int dga = (int)(__ldg(G.offs + a + 1) - __ldg(G.offs + a));
+                        ea[j] = a;
+                        xa[j] = dga;
+                        ya[j] = __ldg(sup + e);
+                        if (W.degfilter && dga < C.mindeg0) Lt = 0;
+                        if (ya[j] == 0) Lt = 0;          // no triangle on (a, b)
+                    } else {
+                        ea[j] = e;
+                        xa[j] = 0;
                     }
                 }
+                int x = Lt;                       // inclusive warp scan
+    #pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const int y = __shfl_up_sync(FULLMASK, x, o);
+                    if (lane >= o) x += y;
+                }
+                if (j < len) pre[j] = carry + x - Lt;
+                carry += __shfl_sync(FULLMASK, x, 31);
             }
+            if (lane == 0) pre[len] = carry;
+            __syncwarp();
+            const int total = carry;
+            int lo = 0;                           // monotone: last j with pre[j] <= idx
+            for (int v0 = 0; v0 < total; v0 += 64) {
+                int jj[2], cc[2];
+                uint32_t pp[2];
+                bool ok[2];
+    #pragma unroll
+                for (int r = 0; r < 2; ++r) {
+                    const int idx = v0 + 32 * r + lane;
+                    ok[r] = idx < total;
+                    jj[r] = 0; pp[r] = 0; cc[r] = -1;
+                    if (ok[r]) {
+                        int l2 = lo, hi = len;
+                        while (hi - l2 > 1) {
+                            const int mid = (l2 + hi) >> 1;
+                            if (pre[mid] <= idx) l2 = mid; else hi = mid;
+                        }
+                        lo = l2;
+                        jj[r] = l2;
+                        pp[r] = q0[l2] + (uint32_t)(idx - pre[l2]);
+                        cc[r] = __ldg(G.adj + pp[r]);
+                    }
+                }
+    #pragma unroll
+                for (int r = 0; r < 2; ++r) {
+                    const int h = ok[r] ? hfind(key, cc[r], hbits) : -1;
+                    bool hit = h >= 0;
+                    if (TRI) {
+                        int dw = 0, cvw = 0;
+                        if (hit) {
+                            const int kk = kpos[h];
+                            dw = pay1[kk];
+                            cvw = pay0[kk];
+                            if (W.degfilter && dw < C.mindeg2) hit = false;
+                        }
+                        cnt = tri_append(leaf, cnt, hit, ea[jj[r]], b, cc[r], xa[jj[r]], degb, dw, ya[jj[r]],
+                                         pp[r] - da[jj[r]], cvw, lane);
+                        if (cnt >= 32) {
+                            tri_flush<NP, MODE == 2>(G, H, P, VD, C, sup, leaf, cnt, lrows, blockDim.x, wrows, lane, sa, ZS);
+                            if (lane == 0) nmatch += cnt;
+                            cnt = 0;
+                        }
+                    } else {
+                        const unsigned hmask = __ballot_sync(FULLMASK, hit);
+                        if (hit) {
+                            atomicAdd(&pay0[h], 1);                              // c(bc)
+                            atomicAdd(sup + (pp[r] - da[jj[r]]), 1);             // c(ac)
+                            const unsigned peers = __match_any_sync(hmask, jj[r]);   // c(ab): one add per a
+                            if ((peers & ((1u << lane) - 1)) == 0) atomicAdd(&xa[jj[r]], __popc(peers));
+                        }
+                    }
+                }
+            }
+            __syncwarp();
+            if (!TRI) {
+                for (int j = lane; j < len; j += 32)
+                    if (xa[j]) atomicAdd(sup + ea[j], xa[j]);
+            }
+            __syncwarp();
         }
-        __syncwarp();
-        if (!TRI) {
-            for (int j = lane; j < len; j += 32)
-                if (xa[j]) atomicAdd(sup + ea[j], xa[j]);
-        }
-        __syncwarp();
     }
     if (TRI) {
         if (cnt) {
@@ -688,8 +708,8 @@ __host__ __device__ inline size_t blocktab_table_bytes(int hs, int maxout, bool 
     const size_t b = (size_t)hs * 6 + (tri ? (size_t)maxout * 8 : (size_t)hs * 4);
     return (b + 15) & ~(size_t)15;
 }
-__host__ __device__ inline size_t blocktab_warp_bytes(bool tri) {
-    return tri ? (size_t)kLeafCap * kLeafW * 4 + (size_t)kMaxVennRows * 16 : 0;
+__host__ __device__ inline size_t blocktab_warp_bytes(int mode) {   // leaf buffer (+ Venn warp rows, MODE 1)
+    return mode ? (size_t)kLeafCap * kLeafW * 4 + (mode == 1 ? (size_t)kMaxVennRows * 16 : 0) : 0;
 }
 
 template <int MODE, int NP>
@@ -703,6 +723,7 @@ __global__ void __launch_bounds__((MODE ? kBlockTriWarps : kBlockTabWarps) * 32,
     extern __shared__ __align__(16) unsigned char s_lb[];
     __shared__ long long s_unit;
     __shared__ int s_next;
+    constexpr int kSubC = TRI ? kSubCTri : kSubCSup;
     __shared__ int32_t s_pre[kSubC + 1];          // sub-chunk: exclusive scan of the tail lengths
     __shared__ uint32_t s_q0[kSubC], s_da[kSubC];  // tail start in adj, split[a] - oofs[a]
     __shared__ int32_t s_e[kSubC], s_x[kSubC];     // support: e(ab), c(ab) count | tri-core: a, deg a
@@ -715,10 +736,10 @@ __global__ void __launch_bounds__((MODE ? kBlockTriWarps : kBlockTabWarps) * 32,
     int16_t* kpos = reinterpret_cast<int16_t*>(key + HS);
     int32_t* pay0 = reinterpret_cast<int32_t*>(kpos + HS);   // cnt[slot] | tsup[pos]
     int32_t* pay1 = pay0 + maxout;                            // - | tdeg[pos]
-    unsigned char* wb = s_lb + tab_b + (size_t)w * blocktab_warp_bytes(TRI);
+    unsigned char* wb = s_lb + tab_b + (size_t)w * blocktab_warp_bytes(MODE);
     uint32_t* leaf = reinterpret_cast<uint32_t*>(wb);
     u128* wrows = reinterpret_cast<u128*>(wb + (size_t)kLeafCap * kLeafW * 4);
-    u128* lrows = reinterpret_cast<u128*>(s_lb + tab_b + NWB * blocktab_warp_bytes(TRI)) + tid;
+    u128* lrows = reinterpret_cast<u128*>(s_lb + tab_b + NWB * blocktab_warp_bytes(MODE)) + tid;
 
     __shared__ AccDev s_acc[NWB][TRI ? NP : 1];   // per-warp pattern sums (tri-core)
     __shared__ ZTerm s_zt[TRI ? kZShared : 1];
