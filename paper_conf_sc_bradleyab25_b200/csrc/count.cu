@@ -246,6 +246,7 @@ struct PassExec {
     int kind = 0;              // 0 vertex, 1 edge (support + fc), 2 general core
     int npc = 1;               // accumulator width class
     bool zonly = false;        // triangle cores: Z-term-only listing kernels (no leaf can leave the 128-bit tier)
+    int nwb2 = 8;              // triangle cores: warps per block of the block-table kernel
     int64_t grid = 1;
     size_t smem = 0;
     WorkDesc W{};
@@ -784,9 +785,18 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
             X.grid = std::max<int64_t>(1, std::min<int64_t>((int64_t)nsm * std::min(occ, 16),
                                                             (units_w + kWarpTabWarps - 1) / kWarpTabWarps));
             X.hbits2 = table_hbits(g->sup_maxout);
-            X.smem2 = blocktab_table_bytes(1 << X.hbits2, (int)g->sup_maxout, true) +
-                      kBlockTriWarps * blocktab_warp_bytes(X.zonly ? 2 : 1) + rows;
-            occ = occupancy(tri_kernel(X.zonly, true, X.npc), kBlockTriWarps * 32, X.smem2);
+            // block tables: warps per block with the most resident warps
+            // (Z-only kernel: 8, 12 or 16 -- a large table fits twice per SM
+            // with 12 warps each; MODE 1: 8)
+            {
+                int best = -1;
+                for (int nw : X.zonly ? std::vector<int>{8, 12, 16} : std::vector<int>{kBlockTriWarps}) {
+                    const size_t sm2 = blocktab_table_bytes(1 << X.hbits2, (int)g->sup_maxout, true) +
+                                       nw * blocktab_warp_bytes(X.zonly ? 2 : 1) + rows;
+                    const int o = occupancy(tri_kernel(X.zonly, true, X.npc), nw * 32, sm2);
+                    if (o * nw > best) { best = o * nw; X.nwb2 = nw; X.smem2 = sm2; occ = o; }
+                }
+            }
             if (occ == 0 && units_b > 0)
                 FSGC_FAIL(FSGC_ERR_INVALID, "triangle-core pass: block table of out-degree %lld does not fit "
                           "shared memory (%zu B)", (long long)g->sup_maxout, X.smem2);
@@ -794,8 +804,8 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
                                                              std::max<int64_t>(1, units_b)));
             if (tune("FSGC_VENN_INFO", 0))
                 fprintf(stderr, "[tri] zonly %d; warp tables: %zu B smem, grid %lld; block tables (max out %lld): "
-                        "%zu B smem, %d blocks/SM, grid %lld\n", (int)X.zonly, X.smem, (long long)X.grid,
-                        (long long)g->sup_maxout, X.smem2, occ, (long long)X.grid2);
+                        "%d warps, %zu B smem, %d blocks/SM, grid %lld\n", (int)X.zonly, X.smem, (long long)X.grid,
+                        (long long)g->sup_maxout, X.nwb2, X.smem2, occ, (long long)X.grid2);
             if (X.grid + X.grid2 > (int64_t)nsm * 16)
                 FSGC_FAIL(FSGC_ERR_INTERNAL, "triangle-core pass: block partials overflow");
         }
@@ -926,7 +936,7 @@ extern "C" int fsgc_plan_enqueue_stage(const fsgc_plan* P, void* workspace, void
             else if (X.kind == 3) {
                 if (g->nsup_units_big > 0)
                     FSGC_CUDA(cudaLaunchKernel(tri_kernel(X.zonly, true, X.npc), dim3((unsigned)X.grid2),
-                                               dim3(kBlockTriWarps * 32), args_t2, X.smem2, st));
+                                               dim3(X.nwb2 * 32), args_t2, X.smem2, st));
                 if (g->nsup_units > 0)
                     FSGC_CUDA(cudaLaunchKernel(tri_kernel(X.zonly, false, X.npc), dim3((unsigned)X.grid),
                                                dim3(kWarpTabWarps * 32), args_t, X.smem, st));

@@ -40,11 +40,12 @@
 #define FSGC_ZONLY_MINB 4         // resident blocks per SM the Z-only listing kernels are compiled for
 #endif
 constexpr int kLeafCap = 64;      // leaf buffer per warp (flushed at >= 32)
-constexpr int kLeafW = 10;        // a, b, c, du, dv, dw, cuv, e(ac), cvw, pad
+constexpr int kLeafW = 9;         // a, b, c, du, dv, dw, cuv, e(ac), cvw
 constexpr int kILP = 4;           // tail loads in flight per lane (block tables)
 constexpr int kWarpTabWarps = 8;  // warps per block, warp-table kernels
 constexpr int kBlockTabWarps = 16;   // warps per block, block-table support kernel
-constexpr int kBlockTriWarps = 8;    // warps per block, block-table tri-core kernel
+constexpr int kBlockTriWarps = 8;    // warps per block, block-table tri-core kernel (MODE 1)
+constexpr int kBlockTriWarpsMax = 16;   // Z-only block kernel: 8, 12 or 16 warps (host: most resident warps)
 constexpr int kSubCSup = 512;        // in-entries per concatenated sub-chunk, block-table support kernel
 constexpr int kSubCTri = 256;        // ... tri-core kernel (shared memory: 2 blocks/SM with RMAT-26's table)
 
@@ -237,7 +238,7 @@ __device__ __noinline__ W zterm_sum(int z1, int z2, int z3, int z4, int z5, int 
 // the pass's Z-term table staged in shared memory at kernel start (the flush
 // is out of line, so reading it from the kernel parameters would go through
 // generic loads)
-constexpr int kZShared = 128;
+constexpr int kZShared = 64;
 struct ZShared {
     const ZTerm* terms;          // shared copy (or the global table when it is larger)
     const uint16_t* zoff;        // [FSGC_MAXPATS + 1]
@@ -458,6 +459,31 @@ __device__ __forceinline__ ZShared zshared_stage(const VennDev& VD, ZTerm* s_zt,
     for (int i = tid; i <= FSGC_MAXPATS; i += nthr) s_zoff[i] = VD.zoff[i];
     for (int i = tid; i < FSGC_MAXPATS; i += nthr) s_z64[i] = VD.zmax64p[i];
     return ZShared{fits ? s_zt : VD.zterms, s_zoff, s_z64};
+}
+
+// end of a triangle-core kernel: the warps' shared pattern sums and match
+// counts summed by warp 0, one 128-bit atomic per pattern into the pass
+// result (the triangle-core sink is always in atomic mode)
+template <int NP>
+__device__ __forceinline__ void sacc_publish(AccDev (*s_acc)[NP], unsigned long long* s_nm, int nwb,
+                                             unsigned long long nmatch, const Sink& S, int w, int lane) {
+    if (lane == 0) s_nm[w] = nmatch;
+    __syncthreads();
+    if (w != 0) return;
+    for (int p = lane; p < NP; p += 32) {
+        u128 v = 0;
+        bool o = false;
+        for (int q = 0; q < nwb; ++q) {
+            v = add_ovf(v, u128_make(s_acc[q][p].lo, s_acc[q][p].hi), o);
+            o = o || s_acc[q][p].ovf;
+        }
+        if (v != 0 || o) atomic_add_u128(S.acc + p, v, o);
+    }
+    if (lane == 0) {
+        unsigned long long nm = 0;
+        for (int q = 0; q < nwb; ++q) nm += s_nm[q];
+        if (nm) atomicAdd(S.matches, nm);
+    }
 }
 
 // the warp's shared pattern sums as lane 0's register accumulators (for the
@@ -691,7 +717,8 @@ __global__ void __launch_bounds__(kWarpTabWarps * 32, MODE == 2 ? FSGC_ZONLY_MIN
             tri_flush<NP, MODE == 2>(G, H, P, VD, C, sup, leaf, cnt, lrows, blockDim.x, wrows, lane, sa, ZS);
             if (lane == 0) nmatch += cnt;
         }
-        block_publish<NP>(sacc_to_lane0<NP>(s_acc[w], lane), nmatch, S);
+        __shared__ unsigned long long s_nm[kWarpTabWarps];
+        sacc_publish<NP>(s_acc, s_nm, kWarpTabWarps, nmatch, S, w, lane);
     } else if (prev_b >= 0) {
         __syncwarp();
         table_flush(O, sup, prev_b, hbits, key, kpos, pay0, lane, 32);
@@ -713,13 +740,15 @@ __host__ __device__ inline size_t blocktab_warp_bytes(int mode) {   // leaf buff
 }
 
 template <int MODE, int NP>
-__global__ void __launch_bounds__((MODE ? kBlockTriWarps : kBlockTabWarps) * 32, MODE == 2 ? FSGC_ZONLY_MINB : MODE)
+__global__ void __launch_bounds__((MODE == 1 ? kBlockTriWarps : MODE == 2 ? kBlockTriWarpsMax : kBlockTabWarps) * 32,
+                                  MODE == 2 ? 2 : MODE)
     list_block_kernel(
     GraphDev G, OrientDev O, HubDev H, const int32_t* __restrict__ rev, const uint64_t* __restrict__ units,
     int64_t nunits, int hbits_max, int maxout, int* __restrict__ sup, unsigned long long* queue, int shard, int nshards,
     const __grid_constant__ CoreProg P, WorkDesc W, const __grid_constant__ VennDev VD, const Sink S) {
     constexpr bool TRI = MODE != 0;
-    constexpr int NWB = TRI ? kBlockTriWarps : kBlockTabWarps;
+    constexpr int NWBMAX = MODE == 1 ? kBlockTriWarps : MODE == 2 ? kBlockTriWarpsMax : kBlockTabWarps;
+    const int NWB = blockDim.x >> 5;   // (MODE 2: the host's choice, <= NWBMAX)
     extern __shared__ __align__(16) unsigned char s_lb[];
     __shared__ long long s_unit;
     __shared__ int s_next;
@@ -728,7 +757,7 @@ __global__ void __launch_bounds__((MODE ? kBlockTriWarps : kBlockTabWarps) * 32,
     __shared__ uint32_t s_q0[kSubC], s_da[kSubC];  // tail start in adj, split[a] - oofs[a]
     __shared__ int32_t s_e[kSubC], s_x[kSubC];     // support: e(ab), c(ab) count | tri-core: a, deg a
     __shared__ int32_t s_y[TRI ? kSubC : 1];       // tri-core: c(ab)
-    __shared__ int32_t s_wsum[NWB];
+    __shared__ int32_t s_wsum[kSubC / 32];
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, tid = threadIdx.x, nthr = blockDim.x;
     const int HS = 1 << hbits_max;
     const size_t tab_b = blocktab_table_bytes(HS, maxout, TRI);
@@ -741,11 +770,11 @@ __global__ void __launch_bounds__((MODE ? kBlockTriWarps : kBlockTabWarps) * 32,
     u128* wrows = reinterpret_cast<u128*>(wb + (size_t)kLeafCap * kLeafW * 4);
     u128* lrows = reinterpret_cast<u128*>(s_lb + tab_b + NWB * blocktab_warp_bytes(MODE)) + tid;
 
-    __shared__ AccDev s_acc[NWB][TRI ? NP : 1];   // per-warp pattern sums (tri-core)
+    __shared__ AccDev s_acc[TRI ? NWBMAX : 1][TRI ? NP : 1];   // per-warp pattern sums (tri-core)
     __shared__ ZTerm s_zt[TRI ? kZShared : 1];
     __shared__ uint16_t s_zoff[FSGC_MAXPATS + 1];
     __shared__ int32_t s_z64[FSGC_MAXPATS];
-    const SAcc sa{s_acc[w]};
+    const SAcc sa{s_acc[TRI ? w : 0]};
     if (TRI && lane < NP) s_acc[w][lane] = AccDev{0, 0, 0, 0, 0};
     ZShared ZS{nullptr, nullptr, nullptr};
     if (TRI) ZS = zshared_stage(VD, s_zt, s_zoff, s_z64, tid, nthr);
@@ -821,11 +850,11 @@ __global__ void __launch_bounds__((MODE ? kBlockTriWarps : kBlockTabWarps) * 32,
             }
             if (tid == 0) s_next = 0;
             __syncthreads();
-            {   // exclusive scan of s_pre[0, kSubC): a segment per warp, then the warp offsets
-                constexpr int segL = kSubC / NWB;
-                int run = 0;
-                for (int c0 = 0; c0 < segL; c0 += 32) {
-                    const int j = w * segL + c0 + lane;
+            {   // exclusive scan of s_pre[0, kSubC): 32-entry segments over the
+                // warps (warp scans), then the segment offsets
+                constexpr int NSEG = kSubC / 32;
+                for (int sg = w; sg < NSEG; sg += NWB) {
+                    const int j = sg * 32 + lane;
                     const int v = s_pre[j];
                     int x = v;
 #pragma unroll
@@ -833,15 +862,16 @@ __global__ void __launch_bounds__((MODE ? kBlockTriWarps : kBlockTabWarps) * 32,
                         const int y = __shfl_up_sync(FULLMASK, x, o);
                         if (lane >= o) x += y;
                     }
-                    s_pre[j] = run + x - v;
-                    run += __shfl_sync(FULLMASK, x, 31);
+                    s_pre[j] = x - v;
+                    if (lane == 31) s_wsum[sg] = x;
                 }
-                if (lane == 0) s_wsum[w] = run;
                 __syncthreads();
-                int off = 0;
-                for (int q = 0; q < w; ++q) off += s_wsum[q];
-                for (int c0 = 0; c0 < segL; c0 += 32) s_pre[w * segL + c0 + lane] += off;
-                if (w == NWB - 1 && lane == 0) s_pre[kSubC] = off + run;
+                for (int sg = w; sg < NSEG; sg += NWB) {
+                    int off = 0;
+                    for (int q = 0; q < sg; ++q) off += s_wsum[q];
+                    s_pre[sg * 32 + lane] += off;
+                    if (sg == NSEG - 1 && lane == 31) s_pre[kSubC] = off + s_wsum[sg];
+                }
                 __syncthreads();
             }
             const int total = s_pre[kSubC];
@@ -915,7 +945,8 @@ __global__ void __launch_bounds__((MODE ? kBlockTriWarps : kBlockTabWarps) * 32,
             tri_flush<NP, MODE == 2>(G, H, P, VD, C, sup, leaf, cnt, lrows, nthr, wrows, lane, sa, ZS);
             if (lane == 0) nmatch += cnt;
         }
-        block_publish<NP>(sacc_to_lane0<NP>(s_acc[w], lane), nmatch, S);
+        __shared__ unsigned long long s_nm[NWBMAX];
+        sacc_publish<NP>(s_acc, s_nm, NWB, nmatch, S, w, lane);
     } else if (cur_b >= 0) {
         table_flush(O, sup, cur_b, hbits, key, kpos, pay0, tid, nthr);
     }
