@@ -207,6 +207,25 @@ __device__ __forceinline__ W binom_fly(uint64_t n, int j) {
     for (int i = 2; i <= j; ++i) c = ((c * (W)(n - (uint64_t)i + 1)) >> c_tz[i]) * inv_odd(i, c);
     return c;
 }
+// 64-bit tier, the common small case: j <= 4 and n < 2^16 by the products
+// n(n-1)(n-2)(n-3) < 2^64 in 32-bit pieces and one exact division (a shift
+// for the 2-power, the inverse of 3 mod 2^64 for the odd part); the factors
+// vanish for n < j as in the chain
+template <>
+__device__ __forceinline__ uint64_t binom_fly<uint64_t>(uint64_t n, int j) {
+    if (n < 65536u && j <= 4) {
+        const uint32_t m = (uint32_t)n;
+        const uint32_t a = m * (m - 1u);                     // < 2^32
+        if (j <= 1) return j == 1 ? n : 1u;
+        if (j == 2) return a >> 1;
+        const uint64_t inv3 = 0xAAAAAAAAAAAAAAABull;
+        if (j == 3) return (((uint64_t)a * (uint64_t)(m - 2u)) >> 1) * inv3;
+        return (((uint64_t)a * (uint64_t)(uint32_t)((m - 2u) * (m - 3u))) >> 3) * inv3;
+    }
+    uint64_t c = n;
+    for (int i = 2; i <= j; ++i) c = ((c * (n - (uint64_t)i + 1)) >> c_tz[i]) * c_inv_odd[i];
+    return c;
+}
 
 // one pattern's terms [t0, t1) of the Z-term table on one triangle, mod
 // 2^bits(W).  Out of line: one copy per tier, called once per (leaf, pattern)
