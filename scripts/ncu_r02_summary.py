@@ -32,8 +32,30 @@ def short(name):
 
 def main():
     tag, wl, path = sys.argv[1], sys.argv[2], sys.argv[3]
-    rows = list(csv.reader(open(path)))
-    h = rows[0]
+    txt = open(path).read()
+    if '"Metric Name"' in txt:          # --metrics --csv (long format): pivot to one row per launch
+        import io
+        body = txt[txt.index('"ID"'):]
+        lr = list(csv.reader(io.StringIO(body)))
+        hc = {c: i for i, c in enumerate(lr[0])}
+        launches, order, mets, munit = {}, [], [], {}
+        for r in lr[1:]:
+            if len(r) < len(lr[0]):
+                continue
+            key = r[hc["ID"]]
+            if key not in launches:
+                launches[key] = {"Kernel Name": r[hc["Kernel Name"]]}
+                order.append(key)
+            mn = r[hc["Metric Name"]]
+            launches[key][mn] = r[hc["Metric Value"]]
+            munit[mn] = r[hc["Metric Unit"]]
+            if mn not in mets:
+                mets.append(mn)
+        h = ["Kernel Name"] + mets
+        rows = [h, [""] + [munit[m] for m in mets]] + [[launches[k].get(c, "") for c in h] for k in order]
+    else:
+        rows = list(csv.reader(io.StringIO(txt))) if False else list(csv.reader(open(path)))
+        h = rows[0]
     units = rows[1]
     col = {c: i for i, c in enumerate(h)}
     name_col = col.get("Kernel Name")
