@@ -185,19 +185,6 @@ __device__ __forceinline__ uint64_t sext<uint64_t>(int64_t c) { return (uint64_t
 template <>
 __device__ __forceinline__ u128 sext<u128>(int64_t c) { return (u128)(__int128)c; }
 
-// Z[cm] of one triangle leaf by core-position mask (a select chain: no
-// dynamic indexing)
-__device__ __forceinline__ uint64_t zsel(int z1, int z2, int z3, int z4, int z5, int z6, int z7, int cm) {
-    int r = z1;
-    r = cm == 2 ? z2 : r;
-    r = cm == 3 ? z3 : r;
-    r = cm == 4 ? z4 : r;
-    r = cm == 5 ? z5 : r;
-    r = cm == 6 ? z6 : r;
-    r = cm == 7 ? z7 : r;
-    return (uint64_t)r;
-}
-
 // C(n, j) mod 2^bits(W) by the exact-division chain C(n, i) = C(n, i-1) (n-i+1) / i
 // (division by the odd part of i via its inverse, by the 2-power by a shift);
 // exact when C(n, i) * i fits for every i <= j -- the tier bound of the caller
@@ -230,8 +217,9 @@ __device__ __forceinline__ uint64_t binom_fly<uint64_t>(uint64_t n, int j) {
 // one pattern's terms [t0, t1) of the Z-term table on one triangle, mod
 // 2^bits(W).  Out of line: one copy per tier, called once per (leaf, pattern)
 template <class W>
-__device__ __noinline__ W zterm_sum(int z1, int z2, int z3, int z4, int z5, int z6, int z7, const ZTerm* zt,
-                                    int t0, int t1) {
+__device__ __noinline__ W zterm_sum(const int* z, const ZTerm* zt, int t0, int t1) {
+    // z: the leaf's Z values by core mask in the thread's local memory (one
+    // load per factor at a warp-uniform index instead of a select chain)
     W sum = 0;
     for (int t = t0; t < t1; ++t) {
         const uint4 e = *reinterpret_cast<const uint4*>(zt + t);   // shared (staged) or global
@@ -240,7 +228,7 @@ __device__ __noinline__ W zterm_sum(int z1, int z2, int z3, int z4, int z5, int 
         uint64_t codes = (uint64_t)(e.z >> 16) | ((uint64_t)e.w << 16);   // 8-bit factor codes
         for (int i = 0; i < nf; ++i, codes >>= 8) {
             const int code = (int)(codes & 255);
-            pr *= binom_fly<W>(zsel(z1, z2, z3, z4, z5, z6, z7, code >> 5), code & 31);
+            pr *= binom_fly<W>((uint64_t)z[code >> 5], code & 31);
         }
         sum += pr;
     }
@@ -292,10 +280,10 @@ __device__ __forceinline__ void zterms_eval_warp(bool act, int zmax, const int (
         // per-leaf sum is below 2^119 by the kernel's bound)
         u128 tot;
         if (__all_sync(FULLMASK, !act || zmax <= T.z64[p])) {
-            const uint64_t v = act ? zterm_sum<uint64_t>(z[1], z[2], z[3], z[4], z[5], z[6], z[7], T.terms, t0, t1) : 0;
+            const uint64_t v = act ? zterm_sum<uint64_t>(z, T.terms, t0, t1) : 0;
             tot = warp_sum_limbs<4>((u128)v);      // 32 x < 2^62: the sum fits 67 bits
         } else {
-            const u128 v = act ? zterm_sum<u128>(z[1], z[2], z[3], z[4], z[5], z[6], z[7], T.terms, t0, t1) : 0;
+            const u128 v = act ? zterm_sum<u128>(z, T.terms, t0, t1) : 0;
             tot = warp_sum_limbs<8>(v);            // 32 x < 2^119 < 2^128
         }
         if (lane == 0 && tot != 0) {
