@@ -786,11 +786,11 @@ extern "C" int fsgc_plan_create(const fsgc_graph* g, const fsgc_pattern* const* 
                                                             (units_w + kWarpTabWarps - 1) / kWarpTabWarps));
             X.hbits2 = table_hbits(g->sup_maxout);
             // block tables: warps per block with the most resident warps
-            // (Z-only kernel: 8, 12 or 16 -- a large table fits twice per SM
+            // (Z-only kernel: 8 or 12 -- a large table fits twice per SM
             // with 12 warps each; MODE 1: 8)
             {
                 int best = -1;
-                for (int nw : X.zonly ? std::vector<int>{8, 12, 16} : std::vector<int>{kBlockTriWarps}) {
+                for (int nw : X.zonly ? std::vector<int>{8, 12} : std::vector<int>{kBlockTriWarps}) {
                     const size_t sm2 = blocktab_table_bytes(1 << X.hbits2, (int)g->sup_maxout, true) +
                                        nw * blocktab_warp_bytes(X.zonly ? 2 : 1) + rows;
                     const int o = occupancy(tri_kernel(X.zonly, true, X.npc), nw * 32, sm2);

@@ -45,7 +45,8 @@ constexpr int kILP = 4;           // tail loads in flight per lane (block tables
 constexpr int kWarpTabWarps = 8;  // warps per block, warp-table kernels
 constexpr int kBlockTabWarps = 16;   // warps per block, block-table support kernel
 constexpr int kBlockTriWarps = 8;    // warps per block, block-table tri-core kernel (MODE 1)
-constexpr int kBlockTriWarpsMax = 16;   // Z-only block kernel: 8, 12 or 16 warps (host: most resident warps)
+constexpr int kBlockTriWarpsMax = 12;   // Z-only block kernel: 8 or 12 warps (host: most resident warps);
+                                        // compiled for 2 blocks of 12 warps: up to 80 registers, no spills
 constexpr int kSubCSup = 512;        // in-entries per concatenated sub-chunk, block-table support kernel
 constexpr int kSubCTri = 256;        // ... tri-core kernel (shared memory: 2 blocks/SM with RMAT-26's table)
 
