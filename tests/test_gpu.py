@@ -545,6 +545,25 @@ def _one_count_subprocess(wl, names, env_extra):
     return {k: v[0] for k, v in d.items()}
 
 
+@pytest.mark.parametrize("knob", ["FSGC_NO_ZONLY", "FSGC_NO_Z_TERMS"])
+def test_triangle_core_fc_paths_agree_rmat18(knob):
+    """configs[4]'s pattern set on RMAT-18 (hubs of degree ~25k: both the 64-
+    and 128-bit tiers of the Z-term path): the Z-only kernels (default), the
+    general triangle-core kernels on the Z path (FSGC_NO_ZONLY=1) and the
+    Venn-term / Listing 5 path (FSGC_NO_Z_TERMS=1) give identical counts;
+    the k-tailed members also equal the edge-core decomposition of the same
+    pattern (independent kernels: support pass + Sec. 3.1 closed form)."""
+    from inputs.patterns import CONFIG_PATTERNS
+    names = CONFIG_PATTERNS["rmat26"]
+    base = _one_count_subprocess("rmat18x", names, {})
+    other = _one_count_subprocess("rmat18x", names, {knob: "1"})
+    assert base == other
+    edge = _one_count_subprocess("rmat18x", ["triangle"] + [f"{k}-tailed-triangle" for k in (2, 3, 4)], {})
+    assert base["triangle/tricore"] == edge["triangle"]
+    for k in (2, 3, 4):
+        assert base[f"{k}-tailed-triangle/tricore"] == edge[f"{k}-tailed-triangle"], k
+
+
 def test_rmat26_full_size_wedge_hash_equals_merge():
     """configs[4] graph at full size (RMAT-26, 1.05e9 distinct edges): the
     triangle and k-tailed-triangle counts of the bench path (wedge-hash
