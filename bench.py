@@ -59,13 +59,16 @@ WORKLOAD_DESC = {
                 "124,651 V / 193,620 E (BASELINE configs[1])",
     "pl2k": "tailed triangle on synthetic power-law graph 2,000 V / 10,000 E (configs[0])",
     "rmat22": "triangle, diamond and k-tailed triangles (k=1..4) on RMAT scale 22 (configs[2] graph)",
+    "rmat22-tri": "the configs[4] triangle-core set (core forced to the triangle, 7 patterns) on RMAT scale 22 "
+                  "(configs[2] graph)",
     "rmat16": "4-clique cores with 1-6 and a diamond core with 1 mixed fringe on RMAT scale 16 "
               "(configs[2] patterns; Table 1's rmat16.sym scale)",
     "pl10m": "Fig. 4 16-vertex/25-edge pattern on synthetic power-law graph, 10M edges (configs[3])",
 }
 
 # per_config block of the default run: (workload, reps per timing)
-PER_CONFIG = [("pl2k", 20), ("internet", 20), ("rmat16", 2), ("rmat22", 3), ("pl10m", 3), ("rmat26-edge", 2)]
+PER_CONFIG = [("pl2k", 20), ("internet", 20), ("rmat16", 2), ("rmat22", 3), ("rmat22-tri", 2), ("pl10m", 3),
+              ("rmat26-edge", 2)]
 
 
 def parse():
@@ -170,7 +173,7 @@ def ncu_traffic(workload, kernel):
 
 
 def graph_key(name):
-    return "rmat26" if name.startswith("rmat26") else name
+    return "rmat26" if name.startswith("rmat26") else "rmat22" if name.startswith("rmat22") else name
 
 
 def load_workload(name, device):

@@ -164,6 +164,10 @@ CONFIG_PATTERNS = {
                "3-tailed-triangle/tricore", "4-tailed-triangle/tricore", "diamond/tricore"],
     # the same patterns decomposed by the Sec. 3.4 heuristic (edge core)
     "rmat26-edge": ["triangle"] + [f"{k}-tailed-triangle" for k in range(1, 5)],
+    # the configs[4] triangle-core set on the configs[2] graph (the headline
+    # pass at a second scale)
+    "rmat22-tri": ["triangle/tricore", "tricore+1f", "tricore+2f", "2-tailed-triangle/tricore",
+                   "3-tailed-triangle/tricore", "4-tailed-triangle/tricore", "diamond/tricore"],
     "rmat26-forced-cores": [f"tricore+{f}f" for f in range(1, 7)] + [f"c4core+{f}f" for f in range(1, 7)],
 }
 

@@ -63,8 +63,8 @@ __device__ __forceinline__ int hfind(const int32_t* key, int x, int hbits) {
 
 // the table of N+(b): keys, kpos = position of the key in N+(b), and the
 // payload, built by `nthr` threads (a warp or a block; the caller
-// synchronises before and after).  Support: cnt[slot] = 0 (the c(b, x)
-// counters).  Tri-core: tsup[i] = c(b, x), tdeg[i] = deg(x) for the i-th
+// synchronises before and after).  Support: cnt[i] = 0 (the c(b, x)
+// counters, by position in N+(b)).  Tri-core: tsup[i] = c(b, x), tdeg[i] = deg(x) for the i-th
 // entry x of N+(b).
 template <bool TRI>
 __device__ __forceinline__ void table_build(const GraphDev& G, const OrientDev& O, const int* __restrict__ sup,
@@ -81,18 +81,18 @@ __device__ __forceinline__ void table_build(const GraphDev& G, const OrientDev& 
             tsup[i] = __ldg(sup + ob0 + i);
             tdeg[i] = (int)(__ldg(G.offs + x + 1) - __ldg(G.offs + x));
         } else {
-            cnt[h] = 0;
+            cnt[i] = 0;
         }
     }
 }
 
-// support: add the table's c(b, x) counters to the support array
-__device__ __forceinline__ void table_flush(const OrientDev& O, int* __restrict__ sup, int b, int hbits,
-                                            const int32_t* key, const int16_t* kpos, const int32_t* cnt, int tid,
-                                            int nthr) {
+// support: add the table's c(b, x) counters (by position in N+(b)) to the
+// support array -- the edges (b, x) are consecutive oriented indices
+__device__ __forceinline__ void table_flush(const OrientDev& O, int* __restrict__ sup, int b, int ob,
+                                            const int32_t* cnt, int tid, int nthr) {
     const int64_t base = __ldg(O.oofs + b);
-    for (int h = tid; h < (1 << hbits); h += nthr)
-        if (key[h] != -1 && cnt[h]) atomicAdd(sup + base + kpos[h], cnt[h]);
+    for (int i = tid; i < ob; i += nthr)
+        if (cnt[i]) atomicAdd(sup + base + i, cnt[i]);
 }
 
 // ------------------------------------------------------------------------
@@ -535,7 +535,7 @@ struct WarpTabLayout {
     static constexpr int HS = 2 * FSGC_SUP_CAPW;
     static constexpr size_t key_b = (size_t)HS * 4;
     static constexpr size_t kpos_b = (size_t)HS * 2;
-    static constexpr size_t pay_b = TRI ? (size_t)FSGC_SUP_CAPW * 8 : (size_t)HS * 4;   // tsup+tdeg | cnt
+    static constexpr size_t pay_b = TRI ? (size_t)FSGC_SUP_CAPW * 8 : (size_t)FSGC_SUP_CAPW * 4;   // tsup+tdeg | cnt
     static constexpr size_t slice_b = (size_t)(kWSub + 4) * 4 + (size_t)5 * kWSub * 4;
     static constexpr size_t leaf_b = TRI ? (size_t)kLeafCap * kLeafW * 4 : 0;
     static constexpr size_t rows_b = MODE == 1 ? (size_t)kMaxVennRows * 16 : 0;     // warp-mode term rows
@@ -598,7 +598,7 @@ __global__ void __launch_bounds__(kWarpTabWarps * 32, MODE == 2 ? FSGC_ZONLY_MIN
         if (b != prev_b) {                    // (re)build the table of N+(b)
             if (!TRI && prev_b >= 0) {
                 __syncwarp();
-                table_flush(O, sup, prev_b, hbits, key, kpos, pay0, lane, 32);
+                table_flush(O, sup, prev_b, ob, pay0, lane, 32);
             }
             const int64_t ob_ = __ldg(G.offs + b);
             sb = __ldg(O.split + b);
@@ -704,7 +704,7 @@ __global__ void __launch_bounds__(kWarpTabWarps * 32, MODE == 2 ? FSGC_ZONLY_MIN
                     } else {
                         const unsigned hmask = __ballot_sync(FULLMASK, hit);
                         if (hit) {
-                            atomicAdd(&pay0[h], 1);                              // c(bc)
+                            atomicAdd(&pay0[kpos[h]], 1);                        // c(bc)
                             atomicAdd(sup + (pp[r] - da[jj[r]]), 1);             // c(ac)
                             const unsigned peers = __match_any_sync(hmask, jj[r]);   // c(ab): one add per a
                             if ((peers & ((1u << lane) - 1)) == 0) atomicAdd(&xa[jj[r]], __popc(peers));
@@ -729,7 +729,7 @@ __global__ void __launch_bounds__(kWarpTabWarps * 32, MODE == 2 ? FSGC_ZONLY_MIN
         sacc_publish<NP>(s_acc, s_nm, kWarpTabWarps, nmatch, S, w, lane);
     } else if (prev_b >= 0) {
         __syncwarp();
-        table_flush(O, sup, prev_b, hbits, key, kpos, pay0, lane, 32);
+        table_flush(O, sup, prev_b, ob, pay0, lane, 32);
     }
 }
 
@@ -738,9 +738,9 @@ __global__ void __launch_bounds__(kWarpTabWarps * 32, MODE == 2 ? FSGC_ZONLY_MIN
 // (HS = pow2 >= 2 * max out(b) slots: key + payload), the block's unit and
 // in-neighbour counters, per warp a leaf buffer and term rows (TRI).
 // table bytes for hbits_max / max out(b): key + kpos per slot, then the
-// payload (support: cnt per slot; tri-core: tsup + tdeg per position)
+// payload per position in N+(b) (support: the c(b, x) counts; tri-core: tsup + tdeg)
 __host__ __device__ inline size_t blocktab_table_bytes(int hs, int maxout, bool tri) {
-    const size_t b = (size_t)hs * 6 + (tri ? (size_t)maxout * 8 : (size_t)hs * 4);
+    const size_t b = (size_t)hs * 6 + (size_t)maxout * (tri ? 8 : 4);
     return (b + 15) & ~(size_t)15;
 }
 __host__ __device__ inline size_t blocktab_warp_bytes(int mode) {   // leaf buffer (+ Venn warp rows, MODE 1)
@@ -805,7 +805,7 @@ __global__ void __launch_bounds__((MODE == 1 ? kBlockTriWarps : MODE == 2 ? kBlo
         if (un < 0) break;
         const int b = (int)((unsigned long long)un >> 32), k = (int)(un & 0xffffffffll);
         if (b != cur_b) {                      // (re)build the block's table of N+(b)
-            if (!TRI && cur_b >= 0) table_flush(O, sup, cur_b, hbits, key, kpos, pay0, tid, nthr);
+            if (!TRI && cur_b >= 0) table_flush(O, sup, cur_b, ob, pay0, tid, nthr);
             const int64_t ob_ = __ldg(G.offs + b);
             sb = __ldg(O.split + b);
             ob = (int)(__ldg(G.offs + b + 1) - sb);
@@ -931,7 +931,7 @@ __global__ void __launch_bounds__((MODE == 1 ? kBlockTriWarps : MODE == 2 ? kBlo
                     } else {
                         const unsigned hmask = __ballot_sync(FULLMASK, hit);
                         if (hit) {
-                            atomicAdd(&pay0[h], 1);                        // c(bc)
+                            atomicAdd(&pay0[kpos[h]], 1);                  // c(bc)
                             atomicAdd(sup + (pp[r] - s_da[j]), 1);          // c(ac)
                             const unsigned peers = __match_any_sync(hmask, j);   // c(ab): one add per a
                             if ((peers & ((1u << lane) - 1)) == 0) atomicAdd(&s_x[j], __popc(peers));
@@ -956,6 +956,6 @@ __global__ void __launch_bounds__((MODE == 1 ? kBlockTriWarps : MODE == 2 ? kBlo
         __shared__ unsigned long long s_nm[NWBMAX];
         sacc_publish<NP>(s_acc, s_nm, NWB, nmatch, S, w, lane);
     } else if (cur_b >= 0) {
-        table_flush(O, sup, cur_b, hbits, key, kpos, pay0, tid, nthr);
+        table_flush(O, sup, cur_b, ob, pay0, tid, nthr);
     }
 }
