@@ -215,7 +215,10 @@ def host_csr(n, e):
     return simple_csr_torch(n, e)
 
 
-def oracle_cpu_sample(csr, pats, budget_s, seed=0, max_deg=20000, nroots=None):
+SAMPLE_MAX_DEG = 64    # sampled roots: degree <= this (per-root oracle cost stays bounded on hub-heavy graphs)
+
+
+def oracle_cpu_sample(csr, pats, budget_s, seed=0, max_deg=SAMPLE_MAX_DEG, nroots=None):
     """The unmodified C oracle (oracle.cfast.root_raw_sum_c: every core map
     with the root pattern vertex on the sampled graph vertices, explicit Venn,
     Listing 5; OpenMP on all host cores) on seeded random root vertices of
@@ -274,14 +277,17 @@ def run_reference(args, rank, world):
     # size one step so the whole run stays within a few minutes
     step_budget = max(0.5, 150.0 / max(1, args.steps + args.warmup))
     _, _, nr, _ = oracle_cpu_sample(csr, pats, step_budget, seed=99)
+    # every step repeats the calibrated sample (same seed, same roots): a
+    # bounded, reproducible amount of oracle work per step
     vals, secs, threads = [], [], 1
     for s in range(args.warmup + args.steps):
-        maps, dt, _, threads = oracle_cpu_sample(csr, pats, 0, seed=s, nroots=nr)
+        maps, dt, _, threads = oracle_cpu_sample(csr, pats, 0, seed=99, nroots=nr)
         if s >= args.warmup:
             vals.append(maps)
             secs.append(dt)
     value = sum(vals) / sum(secs)
-    sample = (f"{nr} seeded random root vertices (degree <= 20000) per step x {len(pats)} patterns, "
+    sample = (f"{nr} seeded random root vertices (degree <= {SAMPLE_MAX_DEG}, the same every step) x {len(pats)} "
+              f"patterns, "
               f"C oracle root sums, {threads} OpenMP threads")
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
@@ -663,7 +669,7 @@ def main():
         log(f"cpu baseline: {nr} roots in {secs:.1f} s")
         del csr
         cpu = {"value": maps / secs, "unit": UNIT, "cores": threads, "kind": "oracle",
-               "sample": f"{nr} seeded random root vertices (degree <= 20000) x {len(pats)} patterns "
+               "sample": f"{nr} seeded random root vertices (degree <= {SAMPLE_MAX_DEG}) x {len(pats)} patterns "
                          f"({secs:.1f} s, C oracle root sums: every core map, explicit Venn, Listing 5; "
                          f"{threads} OpenMP threads)"}
     del e_dev
