@@ -308,9 +308,10 @@ def listing_stats(n, e):
     tensor's device): m, sum over oriented edges (a, b) of the tail length of
     N+(a) after b (the listing kernels' streamed elements), and the merge
     kernel's sum of out(a) + out(b)."""
+    import numpy as np
     import torch
-    dev = e.device if hasattr(e, "device") else "cpu"
-    et = e if hasattr(e, "device") else torch.from_numpy(e)
+    et = e if isinstance(e, torch.Tensor) else torch.from_numpy(np.ascontiguousarray(e))
+    dev = et.device
     a = et[:, 0].to(torch.int64)
     b = et[:, 1].to(torch.int64)
     ok = a != b
@@ -336,7 +337,7 @@ def listing_stats(n, e):
     tail = out[u] - (torch.arange(u.numel(), device=dev) - oofs[u]) - 1
     st = {"m": int(u.numel()), "tail": float(tail.sum()), "merge": float((out[u] + out[v]).sum())}
     del u, v, tail, oofs, out, deg, rank
-    if dev != "cpu":
+    if dev.type != "cpu":
         torch.cuda.empty_cache()
     return st
 
