@@ -896,8 +896,17 @@ __global__ void __launch_bounds__((MODE == 1 ? kBlockTriWarps : MODE == 2 ? kBlo
                     const int idx = e0 + 32 * r + lane;
                     jj[r] = 0; pp[r] = 0; cc[r] = -1;
                     if (idx < total) {
-                        int l2 = lo, hi = kSubC;
+                        int l2 = lo;
                         if (s_pre[l2] > idx) l2 = 0;
+                        // galloping from the lane's previous tail (the next
+                        // element is usually in it or close), then bisection
+                        int hi = l2 + 1, step = 1;
+                        while (hi < kSubC && s_pre[hi] <= idx) {
+                            l2 = hi;
+                            step <<= 1;
+                            hi = l2 + step;
+                        }
+                        if (hi > kSubC) hi = kSubC;
                         while (hi - l2 > 1) {
                             const int mid = (l2 + hi) >> 1;
                             if (s_pre[mid] <= idx) l2 = mid; else hi = mid;
